@@ -1,0 +1,111 @@
+"""The parity comparator (oracle/compare.py) accepts an independent correct
+fp32 factorisation (scipy LAPACK sgeqrf/cgeqrf) and rejects plausible bugs."""
+import numpy as np
+import pytest
+import scipy.linalg.lapack as lapack
+
+import bqr_inputs
+import oracle
+from oracle.compare import compare_geqrf, compare_apply, compare_orgqr
+
+
+def _lapack32(A_cm, m):
+    """Factor each matrix with single-precision LAPACK; returns (out_cm, tau)."""
+    batch, n, lda = A_cm.shape
+    out = A_cm.copy()
+    taus = []
+    f = lapack.cgeqrf if np.iscomplexobj(A_cm) else lapack.sgeqrf
+    for b in range(batch):
+        qr, tau, _, info = f(np.asfortranarray(A_cm[b, :, :m].T))
+        assert info == 0
+        out[b, :, :m] = qr.T
+        taus.append(tau)
+    return out, np.array(taus)
+
+
+@pytest.mark.parametrize("m,n,dt", [(8, 8, "f32"), (56, 56, "f32"), (240, 66, "c64"), (33, 20, "c64")])
+def test_accepts_lapack_fp32(m, n, dt):
+    A = bqr_inputs.random_batch(m, n, 20, dt, seed=5)
+    out, tau = _lapack32(A, m)
+    rep = compare_geqrf(A, m, out, tau)
+    assert rep["ok"], rep
+    assert rep["residual_max"] < 1e-6 and rep["orth_max"] < 5e-6
+
+
+def test_rejects_perturbed_r():
+    A = bqr_inputs.random_batch(16, 16, 8, "f32", seed=6)
+    out, tau = _lapack32(A, 16)
+    out[3, 10, 2] *= 1.001  # R[2,10]
+    rep = compare_geqrf(A, 16, out, tau)
+    assert not rep["ok"] and 3 in rep["fail_idx"]
+
+
+def test_rejects_wrong_tau():
+    A = bqr_inputs.random_batch(16, 16, 8, "f32", seed=7)
+    out, tau = _lapack32(A, 16)
+    tau = tau.copy()
+    tau[5, 4] *= 1.01
+    rep = compare_geqrf(A, 16, out, tau)
+    assert not rep["ok"] and 5 in rep["fail_idx"]
+
+
+def test_rejects_unconjugated_update():
+    """A complex factorisation whose trailing update used tau instead of
+    conj(tau) (reading Q9) must fail."""
+    rng = np.random.default_rng(8)
+    m = n = 6
+    A = (rng.standard_normal((m, n)) + 1j * rng.standard_normal((m, n))).astype(np.complex128)
+    R = A.copy()
+    taus = []
+    for i in range(n):
+        alpha = R[i, i]
+        x = R[i + 1:, i]
+        nu = np.sqrt(abs(alpha) ** 2 + np.vdot(x, x).real)
+        beta = -np.copysign(nu, alpha.real)
+        tau = complex((beta - alpha.real) / beta, -alpha.imag / beta)
+        v = np.concatenate([[1.0], x / (alpha - beta)])
+        R[i + 1:, i] = v[1:]
+        R[i, i] = beta
+        C = R[i:, i + 1:]
+        C -= tau * np.outer(v, np.conj(v) @ C)  # BUG: should be conj(tau)
+        taus.append(tau)
+    A_cm = oracle.to_cm(A[None].astype(np.complex64))
+    out_cm = oracle.to_cm(R[None].astype(np.complex64))
+    rep = compare_geqrf(A_cm, m, out_cm, np.array([taus]))
+    assert not rep["ok"]
+
+
+def test_rejects_unjustified_sign_flip():
+    """Flip the sign of row 0 of R and of reflector 0's Householder sign: a
+    valid QR, but LAPACK's sign rule fixes it when |alpha|/nu is large."""
+    A = bqr_inputs.random_batch(5, 5, 1, "f32", seed=9)
+    out, tau = _lapack32(A, 5)
+    logical = np.swapaxes(out, 1, 2).copy()
+    logical[0, 0, :] *= -1  # R row 0 negated: A = (Q D)(D R) still holds only if Q changes too
+    out2 = np.swapaxes(logical, 1, 2).copy()
+    rep = compare_geqrf(A, 5, out2, tau)
+    assert not rep["ok"]
+
+
+def test_zero_matrix_exact():
+    A = np.zeros((2, 4, 4), np.float32)
+    out = A.copy()
+    tau = np.zeros((2, 4), np.float32)
+    assert compare_geqrf(A, 4, out, tau)["ok"]
+    tau[1, 0] = 1e-30
+    assert not compare_geqrf(A, 4, out, tau)["ok"]
+
+
+def test_apply_and_orgqr_comparators():
+    A = bqr_inputs.random_batch(12, 5, 4, "c64", seed=10)
+    out, tau = _lapack32(A, 12)
+    B = bqr_inputs.rhs_batch(12, 2, 4, "c64", seed=10)
+    ref = oracle.apply_qh_cm(out.astype(np.complex128), 12, 5, tau, B)
+    assert compare_apply(out, 12, 5, tau, B, ref.astype(np.complex64))["ok"]
+    bad = ref.copy()
+    bad[1, 0, 3] += 1e-3
+    assert not compare_apply(out, 12, 5, tau, B, bad)["ok"]
+    Q = oracle.orgqr_cm(out.astype(np.complex128), 12, 5, tau)
+    assert compare_orgqr(out, 12, 5, tau, Q.astype(np.complex64))["ok"]
+    Q[0, 1, 1] += 1e-3
+    assert not compare_orgqr(out, 12, 5, tau, Q)["ok"]
