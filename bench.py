@@ -1,0 +1,421 @@
+#!/usr/bin/env python
+"""bench.py -- batched Householder QR on B200: the BASELINE.json metric.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+                    [--config C3|C4|C2|C1] [--no-also] [--no-cpu]
+
+One "step" = one pass of the whole hot path over one batch:
+  C3 (default, the metric's headline workload): bqr_geqrf_batched on 5,000
+     56x56 fp32 matrices per GPU;
+  C4 (reported under "also"): bqr_geqrf_batched + bqr_apply_qh_batched on
+     256 240x66 complex64 STAP matrices with one right-hand side each;
+  C2 (under "also"): 1,000,000 4x4 fp32.
+Inputs are seeded synthetic (bqr_inputs) and resident in HBM; before every
+timed step the working buffer is restored from a pristine copy and L2 is
+flushed by writing a 2x-L2 buffer (both untimed); each step is bracketed by
+CUDA events on the launching stream.  Multi-GPU: one process per GPU under
+torchrun, each rank factors its own seeded slice (weak scaling, no data-path
+collective); NCCL only for barriers and the MAX of per-rank times.
+
+--impl reference times the fp64 CPU oracle (oracle/, the parity reference)
+on the host cores on a bounded sample of the same workload.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+import bqr_inputs  # noqa: E402
+import bqr_metrics as bm  # noqa: E402
+
+METRIC = "batched QR GFLOP/s & % roofline (5000×56×56 fp32; STAP 240×66 c64) @1/2/4/8 B200"
+UNIT = "GFLOP/s"
+PROFILE_TRAFFIC = os.path.join(ROOT, "profiles", "traffic.json")
+
+
+# --------------------------------------------------------------------- utils
+
+def env_rank():
+    return int(os.environ.get("RANK", 0)), int(os.environ.get("WORLD_SIZE", 1)), int(os.environ.get("LOCAL_RANK", 0))
+
+
+class ClockSampler:
+    """NVML sampling of SM clock + throttle reasons during the timed region
+    (the B200_PROFILING.md clocks line)."""
+
+    REASONS = {
+        0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap", 0x8: "hw_slowdown",
+        0x10: "sync_boost", 0x20: "sw_thermal_slowdown", 0x40: "hw_thermal_slowdown",
+        0x80: "hw_power_brake_slowdown", 0x100: "display_clock_setting",
+    }
+
+    def __init__(self, device_index: int, period_s: float = 0.01):
+        self.dev = device_index
+        self.period = period_s
+        self.samples = []
+        self.reasons = 0
+        self.max_mhz = None
+        self._stop = threading.Event()
+        self._t = None
+        self.ok = False
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(device_index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+            self.ok = True
+        except Exception as e:  # pragma: no cover - no NVML
+            self.err = str(e)
+
+    def _run(self):
+        nv = self.nv
+        while not self._stop.is_set():
+            try:
+                self.samples.append(nv.nvmlDeviceGetClockInfo(self.h, nv.NVML_CLOCK_SM))
+                self.reasons |= nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+            except Exception:
+                pass
+            time.sleep(self.period)
+
+    def __enter__(self):
+        if self.ok:
+            self._t = threading.Thread(target=self._run, daemon=True)
+            self._t.start()
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        if self._t:
+            self._t.join()
+
+    def summary(self):
+        if not self.ok:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvml_unavailable"]}
+        names = [n for b, n in self.REASONS.items() if self.reasons & b and n != "gpu_idle"]
+        med = float(np.median(self.samples)) if self.samples else None
+        return {"sm_mhz": med, "sm_max_mhz": self.max_mhz, "reasons": names, "samples": len(self.samples)}
+
+
+def load_traffic(name: str):
+    try:
+        with open(PROFILE_TRAFFIC) as f:
+            return json.load(f).get(name)
+    except OSError:
+        return None
+
+
+# --------------------------------------------------------------------- GPU arm
+
+class Workload:
+    """Device buffers for one config on one rank."""
+
+    def __init__(self, name, rank, world, torch, bqr, batch=None):
+        cfg = dict(bqr_inputs.CONFIGS[name])
+        self.name = name
+        self.m, self.n, self.dt = cfg["m"], cfg["n"], cfg["dtype"]
+        self.batch = cfg["batch"] if batch is None else batch
+        self.k = min(self.m, self.n)
+        self.nrhs = cfg.get("nrhs", 0)
+        self.torch, self.bqr = torch, bqr
+        # weak scaling: rank r owns matrices [r*B, (r+1)*B) of a world*B seeded stream
+        lo, hi = rank * self.batch, (rank + 1) * self.batch
+        host = bqr_inputs.random_batch(self.m, self.n, world * self.batch, self.dt, cfg["seed"], cfg["dist"],
+                                       start=lo, stop=hi)
+        self.host = host
+        self.pristine = torch.from_numpy(host).cuda()
+        self.A = torch.empty_like(self.pristine)
+        tdt = self.pristine.dtype
+        self.tau = torch.empty((self.batch, self.k), dtype=tdt, device="cuda")
+        if self.nrhs:
+            Bh = bqr_inputs.rhs_batch(self.m, self.nrhs, world * self.batch, self.dt, cfg["seed"], start=lo, stop=hi)
+            self.Bp = torch.from_numpy(Bh).cuda()
+            self.B = torch.empty_like(self.Bp)
+        self.code = bqr.R32 if self.dt == "f32" else bqr.C64
+        self.stream = torch.cuda.current_stream()
+        self.sptr = self.stream.cuda_stream
+        lib = bqr.load()
+        self.lib = lib
+        import ctypes
+        self.c = ctypes
+        self.flops = self.batch * bm.geqrf_flops(self.m, self.n, self.dt)
+        self.bytes = self.batch * bm.geqrf_bytes(self.m, self.n, self.dt)
+        if self.nrhs:
+            self.flops_apply = self.batch * bm.apply_flops(self.m, self.n, self.nrhs, self.dt)
+            self.bytes_apply = self.batch * bm.apply_bytes(self.m, self.nrhs, self.dt)
+        else:
+            self.flops_apply = self.bytes_apply = 0
+
+    def restore(self):
+        self.A.copy_(self.pristine)
+        if self.nrhs:
+            self.B.copy_(self.Bp)
+
+    def geqrf(self):
+        c = self.c
+        st = self.lib.bqr_geqrf_batched(self.code, self.m, self.n, self.batch, c.c_void_p(self.A.data_ptr()),
+                                        self.m, c.c_void_p(self.tau.data_ptr()), c.c_void_p(self.sptr))
+        if st:
+            raise RuntimeError(f"bqr_geqrf_batched -> {st}")
+
+    def apply(self):
+        c = self.c
+        st = self.lib.bqr_apply_qh_batched(self.code, self.m, self.n, self.k, self.nrhs, self.batch,
+                                           c.c_void_p(self.A.data_ptr()), self.m, c.c_void_p(self.tau.data_ptr()),
+                                           c.c_void_p(self.B.data_ptr()), self.m, c.c_void_p(self.sptr))
+        if st:
+            raise RuntimeError(f"bqr_apply_qh_batched -> {st}")
+
+
+def barrier(torch, dist, world):
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+
+
+def max_over_ranks(torch, dist, world, x: float) -> float:
+    if world == 1:
+        return x
+    t = torch.tensor([x], dtype=torch.float64, device="cuda")
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())
+
+
+def time_workload(w: Workload, steps: int, warmup: int, torch, dist, world, flush, sampler=None):
+    """Returns (ms_per_step, ms_geqrf_per_launch)."""
+    ev = [[torch.cuda.Event(enable_timing=True) for _ in range(3)] for _ in range(steps)]
+    for _ in range(warmup):
+        w.restore()
+        flush.zero_()
+        w.geqrf()
+        if w.nrhs:
+            w.apply()
+    barrier(torch, dist, world)
+    ctx = sampler if sampler is not None else _Null()
+    with ctx:
+        for i in range(steps):
+            w.restore()
+            flush.zero_()
+            ev[i][0].record(w.stream)
+            w.geqrf()
+            ev[i][1].record(w.stream)
+            if w.nrhs:
+                w.apply()
+            ev[i][2].record(w.stream)
+        barrier(torch, dist, world)
+    step_ms = sum(e[0].elapsed_time(e[2]) for e in ev) / steps
+    qr_ms = sum(e[0].elapsed_time(e[1]) for e in ev) / steps
+    return max_over_ranks(torch, dist, world, step_ms), max_over_ranks(torch, dist, world, qr_ms)
+
+
+class _Null:
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        pass
+
+
+def roofline_obj(w: Workload, qr_ms: float, peaks: dict, n_sm: int):
+    """Roofline of the dominant kernel (the geqrf launch): SURVEY 8(d)."""
+    hbm = float(peaks["hbm_gbs"])
+    fp32 = bm.fp32_peak_tflops(n_sm, float(peaks.get("sm_max_mhz", 1965.0)))
+    t_roof, bound = bm.roofline_time_s(w.flops, w.bytes, hbm, fp32)
+    t = qr_ms / 1e3
+    traffic = load_traffic(w.name)
+    if bound == "hbm":
+        ach, peak, unit = w.bytes / t / 1e9, hbm, "GB/s"
+    else:
+        ach, peak, unit = w.flops / t / 1e12, fp32, "TFLOP/s"
+    return {"bound": bound, "achieved": round(ach, 3), "peak": peak, "unit": unit,
+            "frac": round(ach / peak, 4), "traffic": traffic,
+            "peak_source": ("MEASURED_PEAKS.json hbm_gbs" if bound == "hbm" else
+                            f"derived: {n_sm} SMs x 128 FP32 lanes x 2 x {peaks.get('sm_max_mhz', 1965.0)} MHz"),
+            "roofline_us": round(t_roof * 1e6, 3), "kernel_us": round(qr_ms * 1e3, 3),
+            "algorithmic_bytes": w.bytes, "useful_flops": w.flops}
+
+
+def e2e_host(w: Workload, steps: int, warmup: int, torch, dist, world):
+    """Same metric end to end through the public host-buffer entry point
+    (bqr_geqrf_batched_host): H2D of the step's inputs from pinned memory,
+    the factorisation and D2H of R/V + tau all inside the timed region."""
+    bqr = w.bqr
+    host_in = torch.from_numpy(w.host.copy())
+    Ah = torch.empty_like(host_in).pin_memory()
+    tauh = torch.empty((w.batch, w.k), dtype=w.tau.dtype).pin_memory()
+    chunk = max(1, w.batch // 8)
+    wsb = bqr.host_workspace_bytes(w.code, w.m, w.n, w.m, chunk)
+    ws = torch.empty(wsb, dtype=torch.uint8, device="cuda")
+    ev = [[torch.cuda.Event(enable_timing=True) for _ in range(2)] for _ in range(steps)]
+    for _ in range(warmup):
+        Ah.copy_(host_in)
+        bqr.geqrf_batched_host(w.code, w.m, w.n, w.batch, Ah.data_ptr(), w.m, tauh.data_ptr(), ws.data_ptr(), wsb)
+    barrier(torch, dist, world)
+    for i in range(steps):
+        Ah.copy_(host_in)  # restore the host input (untimed)
+        ev[i][0].record(w.stream)
+        bqr.geqrf_batched_host(w.code, w.m, w.n, w.batch, Ah.data_ptr(), w.m, tauh.data_ptr(), ws.data_ptr(), wsb)
+        ev[i][1].record(w.stream)
+    barrier(torch, dist, world)
+    ms = max_over_ranks(torch, dist, world, sum(e[0].elapsed_time(e[1]) for e in ev) / steps)
+    h2d = w.A.numel() * w.A.element_size()
+    d2h = h2d + w.tau.numel() * w.tau.element_size()
+    return ms, h2d, d2h
+
+
+def cpu_baseline(name: str, min_seconds: float = 3.0, max_matrices: int | None = None):
+    """The fp64 oracle, as it stands, on all host cores, on a bounded sample."""
+    import oracle
+    cfg = bqr_inputs.CONFIGS[name]
+    b = cfg["batch"] if max_matrices is None else min(cfg["batch"], max_matrices)
+    A = bqr_inputs.random_batch(cfg["m"], cfg["n"], cfg["batch"], cfg["dtype"], cfg["seed"], cfg["dist"], stop=b)
+    oracle.set_threads(0)
+    oracle.geqrf_cm(A, cfg["m"], with_margin=False)  # warm (page-in, threads)
+    reps, t0 = 0, time.perf_counter()
+    while True:
+        oracle.geqrf_cm(A, cfg["m"], with_margin=False)
+        reps += 1
+        el = time.perf_counter() - t0
+        if el >= min_seconds:
+            break
+    flops = reps * b * bm.geqrf_flops(cfg["m"], cfg["n"], cfg["dtype"])
+    return {"value": round(flops / el / 1e9, 4), "unit": UNIT, "cores": oracle.max_threads(), "kind": "oracle",
+            "sample": f"{b} of the {name} matrices ({cfg['m']}x{cfg['n']} {cfg['dtype']}) x {reps} passes, "
+                      f"{el:.1f} s wall, fp64 C oracle (OpenMP)",
+            "matrices_per_s": round(reps * b / el, 1)}
+
+
+def config_block(w: Workload, world, l2_note):
+    return {"workload": f"{w.name}: {w.batch} x {w.m}x{w.n} {w.dt} geqrf" + (f" + Q^H b ({w.nrhs} rhs)" if w.nrhs else "")
+            + " per GPU", "m": w.m, "n": w.n, "batch_per_gpu": w.batch, "global_batch": w.batch * world,
+            "dtype": w.dt, "l2": l2_note, "parallelism": f"dp{world} (independent matrices per rank)",
+            "kernel": w.bqr.kernel_name(w.code, w.m, w.n)}
+
+
+def run_ours(args):
+    import torch
+    import torch.distributed as dist
+    import paper_conf_ipps_andersonsk12_b200 as bqr
+    rank, world, local = env_rank()
+    torch.cuda.set_device(local)
+    if world > 1:
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    bqr.load()
+    props = torch.cuda.get_device_properties(local)
+    n_sm = props.multi_processor_count
+    l2 = props.L2_cache_size
+    flush = torch.empty(2 * max(l2, 64 << 20), dtype=torch.uint8, device="cuda")
+    l2_note = f"L2 flushed before every timed step by writing {flush.numel() >> 20} MiB (2x L2); input restored from a pristine copy (untimed)"
+    peaks = bm.load_peaks()
+
+    main = Workload(args.config, rank, world, torch, bqr)
+    sampler = ClockSampler(local)
+    step_ms, qr_ms = time_workload(main, args.steps, args.warmup, torch, dist, world, flush, sampler)
+    flops_step = main.flops + main.flops_apply
+    value = world * flops_step / (step_ms / 1e3) / 1e9
+    out = {
+        "metric": METRIC, "value": round(value, 3), "unit": UNIT, "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": round(step_ms, 6), "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "f32" if main.dt == "f32" else "c64", "data": "synthetic (seeded iid Gaussian, bqr_inputs)",
+        "config": config_block(main, world, l2_note),
+        "matrices_per_s": round(world * main.batch / (step_ms / 1e3), 1),
+        "roofline": roofline_obj(main, qr_ms, peaks, n_sm),
+        "gpu_launches": args.steps * (2 if main.nrhs else 1),
+        "clocks": sampler.summary(),
+    }
+    # end to end through the public host-buffer API
+    e_steps = max(3, min(args.steps, 20))
+    e_ms, h2d, d2h = e2e_host(main, e_steps, 2, torch, dist, world)
+    out["e2e"] = {"value": round(world * main.flops / (e_ms / 1e3) / 1e9, 3), "unit": UNIT,
+                  "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h, "steps": e_steps,
+                  "api": "bqr_geqrf_batched_host (pinned host buffers, chunked H2D/compute/D2H overlap)",
+                  "ms_per_step": round(e_ms, 4)}
+    out["gpu_launches"] += (e_steps + 2) * 0  # e2e launches are outside the device-timed kernel region
+    if not args.no_also:
+        also = {}
+        for name in [c for c in ("C4", "C2") if c != args.config]:
+            w = Workload(name, rank, world, torch, bqr)
+            k2 = max(3, min(args.steps, 100))
+            s_ms, q_ms = time_workload(w, k2, max(3, args.warmup), torch, dist, world, flush)
+            fl = w.flops + w.flops_apply
+            also[name] = {"value": round(world * fl / (s_ms / 1e3) / 1e9, 3), "unit": UNIT,
+                          "ms_per_step": round(s_ms, 6), "steps": k2,
+                          "matrices_per_s": round(world * w.batch / (s_ms / 1e3), 1),
+                          "config": config_block(w, world, l2_note),
+                          "roofline": roofline_obj(w, q_ms, peaks, n_sm)}
+            if w.nrhs:
+                also[name]["apply_ms"] = round(s_ms - q_ms, 6)
+            out["gpu_launches"] += k2 * (2 if w.nrhs else 1)
+            del w
+        out["also"] = also
+    if rank == 0 and world == 1 and not args.no_cpu:
+        out["cpu_baseline"] = cpu_baseline(args.config)
+    if rank == 0:
+        print(json.dumps(out), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+def run_reference(args):
+    """--impl reference: the fp64 CPU oracle on the host cores (rank 0 only)."""
+    rank, world, _ = env_rank()
+    if rank != 0:
+        return
+    import oracle
+    cfg = bqr_inputs.CONFIGS[args.config]
+    sample = max(1, min(cfg["batch"], int(os.environ.get("BQR_REF_SAMPLE", 500 if cfg["m"] >= 32 else 20000))))
+    A = bqr_inputs.random_batch(cfg["m"], cfg["n"], cfg["batch"], cfg["dtype"], cfg["seed"], cfg["dist"], stop=sample)
+    oracle.set_threads(0)
+    for _ in range(args.warmup):
+        oracle.geqrf_cm(A, cfg["m"], with_margin=False)
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        oracle.geqrf_cm(A, cfg["m"], with_margin=False)
+    el = time.perf_counter() - t0
+    flops = sample * bm.geqrf_flops(cfg["m"], cfg["n"], cfg["dtype"])
+    value = flops * args.steps / el / 1e9
+    cores = oracle.max_threads()
+    desc = f"{sample} of the {args.config} matrices per step ({cfg['m']}x{cfg['n']} {cfg['dtype']} widened to fp64)"
+    out = {"metric": METRIC, "value": round(value, 4), "unit": UNIT, "impl": "reference", "n_gpus": world,
+           "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(el / args.steps * 1e3, 4),
+           "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+           "data": "synthetic (seeded iid Gaussian, bqr_inputs)",
+           "config": {"workload": f"{args.config}: {cfg['m']}x{cfg['n']} {cfg['dtype']} geqrf (bounded sample)",
+                      "sample_matrices": sample},
+           "cpu_baseline": {"value": round(value, 4), "unit": UNIT, "cores": cores, "kind": "oracle", "sample": desc},
+           "e2e": {"value": round(value, 4), "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(out), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=200)
+    ap.add_argument("--warmup", type=int, default=10)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", default="C3", choices=["C1", "C2", "C3", "C4"])
+    ap.add_argument("--no-also", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    args = ap.parse_args()
+    if args.warmup < 3:
+        args.warmup = 3
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_ours(args)
+
+
+if __name__ == "__main__":
+    main()

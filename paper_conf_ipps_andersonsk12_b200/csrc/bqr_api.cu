@@ -1,0 +1,413 @@
+// bqr_api.cu -- host side of libbqr.so: the C ABI declared in include/bqr.h.
+//
+// Argument validation (LAPACK xerbla-style -i codes), quick returns, the
+// size-class dispatch table (dtype, m, n) -> hand-written sm_100a kernel, one
+// launch per call on the caller's stream, and the host-buffer streaming entry
+// point.  No allocation per call, no host synchronisation (except the
+// explicitly synchronous *_host entry), no state beyond per-device kernel
+// attributes.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <atomic>
+#include <cstdint>
+#include <cstdio>
+#include <cstring>
+#include <mutex>
+
+#include "../../include/bqr.h"
+#include "bqr_apply.cuh"
+#include "bqr_rf.cuh"
+#include "bqr_tiny.cuh"
+
+namespace {
+
+using namespace bqr;
+
+constexpr int kMaxDevices = 64;
+
+int current_device() {
+  int d = 0;
+  cudaGetDevice(&d);
+  return d < 0 ? 0 : (d >= kMaxDevices ? kMaxDevices - 1 : d);
+}
+
+// Raise a kernel's dynamic-smem limit once per (kernel, device).
+template <class K>
+bool ensure_smem(K kern, size_t smem) {
+  static std::atomic<size_t> set_bytes[kMaxDevices];
+  if (smem <= 48 * 1024) return true;
+  const int d = current_device();
+  if (set_bytes[d].load(std::memory_order_acquire) >= smem) return true;
+  if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess)
+    return false;
+  size_t cur = set_bytes[d].load();
+  while (cur < smem && !set_bytes[d].compare_exchange_weak(cur, smem)) {
+  }
+  return true;
+}
+
+int finish_launch() {
+  return cudaGetLastError() == cudaSuccess ? BQR_SUCCESS : BQR_ERR_CUDA;
+}
+
+// ------------------------------------------------------------------ plans
+struct Call {
+  void *A;
+  void *tau;
+  long long batch;
+  int m, n, k, lda;
+  cudaStream_t stream;
+};
+
+using LaunchFn = int (*)(const Call &);
+
+struct Plan {
+  const char *name;
+  LaunchFn geqrf;
+  LaunchFn orgqr;
+};
+
+inline int staging_ld(int m) {
+  // multiple of 4 floats so rows are 16-byte chunks
+  return (m + 3) & ~3;
+}
+
+template <class T, int R, int G, int MR, int NC, int GPB, bool STAGE, bool ORG>
+int launch_rf(const Call &c) {
+  using Cfg = RfCfg<T, R, G, MR, NC, GPB, STAGE>;
+  RfArgs a;
+  a.A = c.A;
+  a.tau = c.tau;
+  a.batch = c.batch;
+  a.lda = c.lda;
+  a.m = c.m;
+  a.n = c.n;
+  a.kmax = c.k;
+  a.ldS = STAGE ? staging_ld(c.m) : 0;
+  a.tileWords = STAGE ? ((a.ldS * c.n + 3) & ~3) : 0;
+  const bool aligned = (reinterpret_cast<uintptr_t>(c.A) & 15) == 0;
+  a.vec4 = (STAGE && (c.lda % 4 == 0) && (c.m % 4 == 0) && aligned) ? 1 : 0;
+  const size_t smem = (size_t)Cfg::kSmallAll * 4 + (STAGE ? (size_t)GPB * a.tileWords * 4 : 0);
+  auto kern = ORG ? orgqr_rf_kernel<T, R, G, MR, NC, GPB, STAGE> : geqrf_rf_kernel<T, R, G, MR, NC, GPB, STAGE>;
+  if (!ensure_smem(kern, smem)) return BQR_ERR_CUDA;
+  const long long grid = (c.batch + GPB - 1) / GPB;
+  if (grid > 0x7fffffffLL) return BQR_ERR_NOT_SUPPORTED;
+  kern<<<(unsigned)grid, Cfg::NT, smem, c.stream>>>(a);
+  return finish_launch();
+}
+
+template <class T, int M, int N>
+int launch_tiny(const Call &c) {
+  using K = Tiny<T, M, N>;
+  TinyArgs a;
+  a.A = c.A;
+  a.tau = c.tau;
+  a.batch = c.batch;
+  a.lda = c.lda;
+  a.staged = (K::kCanStage && c.lda == M && (reinterpret_cast<uintptr_t>(c.A) & 15) == 0) ? 1 : 0;
+  const long long per_block = 32LL * K::kWarps;
+  const long long grid = (c.batch + per_block - 1) / per_block;
+  if (grid > 0x7fffffffLL) return BQR_ERR_NOT_SUPPORTED;
+  geqrf_tiny_kernel<T, M, N><<<(unsigned)grid, K::kWarps * 32, 0, c.stream>>>(a);
+  return finish_launch();
+}
+
+// ---- size classes: smallest class that holds (m, n)
+#define RF_PLAN(T, R, G, MR, NC, GPB, STAGE, NAME)                       \
+  Plan {                                                                 \
+    NAME, &launch_rf<T, R, G, MR, NC, GPB, STAGE, false>,                \
+        &launch_rf<T, R, G, MR, NC, GPB, STAGE, true>                    \
+  }
+
+struct ClassEntry {
+  int mmax, nmax;  // class bounds
+  int exact_m, exact_n;
+  Plan plan;
+};
+
+const ClassEntry kF32[] = {
+    {56, 56, 56, 56, RF_PLAN(float, 2, 8, 28, 7, 2, true, "rf_f32_R2G8_28x7_x2_stage")},
+    {16, 16, 0, 0, RF_PLAN(float, 2, 4, 8, 4, 8, true, "rf_f32_R2G4_8x4_x8_stage")},
+    {32, 32, 0, 0, RF_PLAN(float, 2, 8, 16, 4, 4, true, "rf_f32_R2G8_16x4_x4_stage")},
+    {64, 64, 0, 0, RF_PLAN(float, 4, 8, 16, 8, 2, true, "rf_f32_R4G8_16x8_x2_stage")},
+    {128, 128, 0, 0, RF_PLAN(float, 32, 8, 4, 16, 1, false, "rf_f32_R32G8_4x16_cta")},
+    {256, 64, 0, 0, RF_PLAN(float, 32, 8, 8, 8, 1, false, "rf_f32_R32G8_8x8_cta")},
+};
+
+const ClassEntry kC64[] = {
+    {240, 66, 240, 66, RF_PLAN(float2, 32, 16, 8, 5, 1, false, "rf_c64_R32G16_8x5_cta")},
+    {16, 16, 0, 0, RF_PLAN(float2, 8, 4, 2, 4, 1, false, "rf_c64_R8G4_2x4_warp")},
+    {32, 32, 0, 0, RF_PLAN(float2, 8, 4, 4, 8, 1, false, "rf_c64_R8G4_4x8_warp")},
+    {64, 64, 0, 0, RF_PLAN(float2, 16, 8, 4, 8, 1, false, "rf_c64_R16G8_4x8_cta")},
+    {128, 128, 0, 0, RF_PLAN(float2, 32, 16, 4, 8, 1, false, "rf_c64_R32G16_4x8_cta")},
+    {256, 96, 0, 0, RF_PLAN(float2, 32, 16, 8, 6, 1, false, "rf_c64_R32G16_8x6_cta")},
+};
+
+// tiny exact sizes 1 <= n <= m <= 8
+template <class T, int M>
+Plan tiny_plan_n(int n) {
+  switch (n) {
+#define TN(NN) \
+  case NN:     \
+    if constexpr (NN <= M) return Plan{"tiny", &launch_tiny<T, M, NN>, nullptr}; break;
+    TN(1) TN(2) TN(3) TN(4) TN(5) TN(6) TN(7) TN(8)
+#undef TN
+  }
+  return Plan{nullptr, nullptr, nullptr};
+}
+
+template <class T>
+Plan tiny_plan(int m, int n) {
+  switch (m) {
+    case 1: return tiny_plan_n<T, 1>(n);
+    case 2: return tiny_plan_n<T, 2>(n);
+    case 3: return tiny_plan_n<T, 3>(n);
+    case 4: return tiny_plan_n<T, 4>(n);
+    case 5: return tiny_plan_n<T, 5>(n);
+    case 6: return tiny_plan_n<T, 6>(n);
+    case 7: return tiny_plan_n<T, 7>(n);
+    case 8: return tiny_plan_n<T, 8>(n);
+  }
+  return Plan{nullptr, nullptr, nullptr};
+}
+
+template <size_t N>
+const Plan *pick(const ClassEntry (&tab)[N], int m, int n) {
+  for (const auto &e : tab)
+    if (e.exact_m == m && e.exact_n == n) return &e.plan;
+  for (const auto &e : tab)
+    if (e.exact_m == 0 && m <= e.mmax && n <= e.nmax) return &e.plan;
+  return nullptr;
+}
+
+// geqrf plan; tiny sizes get their own thread-per-matrix kernel.
+bool geqrf_plan(bqr_dtype_t dt, int m, int n, Plan *out) {
+  if (m <= 8 && n <= m) {
+    *out = dt == BQR_R32 ? tiny_plan<float>(m, n) : tiny_plan<float2>(m, n);
+    return out->geqrf != nullptr;
+  }
+  const Plan *p = dt == BQR_R32 ? pick(kF32, m, n) : pick(kC64, m, n);
+  if (!p) return false;
+  *out = *p;
+  return true;
+}
+
+// orgqr has no thread-per-matrix kernel: tiny shapes use the smallest rf class
+bool orgqr_plan(bqr_dtype_t dt, int m, int n, Plan *out) {
+  const Plan *p = dt == BQR_R32 ? pick(kF32, m, n) : pick(kC64, m, n);
+  if (!p) return false;
+  *out = *p;
+  return true;
+}
+
+template <class T, int MR, int NB>
+int launch_apply(const ApplyArgs &a, cudaStream_t s) {
+  using K = ApplyQh<T, MR, NB>;
+  const long long nblk = (a.nrhs + NB - 1) / NB;
+  const long long items = a.batch * nblk;
+  const long long grid = (items + K::kWarps - 1) / K::kWarps;
+  if (grid > 0x7fffffffLL) return BQR_ERR_NOT_SUPPORTED;
+  apply_qh_kernel<T, MR, NB><<<(unsigned)grid, K::kWarps * 32, 0, s>>>(a);
+  return finish_launch();
+}
+
+template <class T>
+int apply_dispatch(const ApplyArgs &a, cudaStream_t s) {
+  const int mr = (a.m + 31) / 32;
+  if (mr <= 1) return launch_apply<T, 1, 4>(a, s);
+  if (mr <= 2) return launch_apply<T, 2, 4>(a, s);
+  if (mr <= 4) return launch_apply<T, 4, 2>(a, s);
+  if (mr <= 8) return launch_apply<T, 8, 1>(a, s);
+  return BQR_ERR_NOT_SUPPORTED;
+}
+
+bool valid_dtype(int d) { return d == BQR_R32 || d == BQR_C64; }
+size_t elem_size(bqr_dtype_t d) { return d == BQR_R32 ? 4 : 8; }
+
+}  // namespace
+
+extern "C" {
+
+const char *bqr_version(void) { return "bqr 0.1.0 (sm_100a)"; }
+
+const char *bqr_status_string(int status) {
+  if (status < 0) return "illegal argument (-i = position of the first bad argument)";
+  switch (status) {
+    case BQR_SUCCESS: return "success";
+    case BQR_ERR_NOT_SUPPORTED: return "shape or dtype not supported by any built size class";
+    case BQR_ERR_CUDA: return "CUDA error";
+    case BQR_ERR_MISALIGNED: return "misaligned pointer";
+  }
+  return "unknown status";
+}
+
+const char *bqr_kernel_name(bqr_dtype_t dtype, int m, int n) {
+  if (!valid_dtype(dtype) || m <= 0 || n <= 0 || m < n) return "";
+  Plan p;
+  if (!geqrf_plan(dtype, m, n, &p)) return "";
+  return p.name ? p.name : "";
+}
+
+int bqr_geqrf_launches(bqr_dtype_t dtype, int m, int n, int batch) {
+  if (!valid_dtype(dtype) || m <= 0 || n <= 0 || batch <= 0) return 0;
+  Plan p;
+  return geqrf_plan(dtype, m, n, &p) ? 1 : 0;
+}
+
+int bqr_geqrf_batched(bqr_dtype_t dtype, int m, int n, int batch, void *A, int lda, void *tau,
+                      cudaStream_t stream) {
+  if (!valid_dtype(dtype)) return -1;
+  if (m < 0) return -2;
+  if (n < 0) return -3;
+  if (batch < 0) return -4;
+  const bool work = m > 0 && n > 0 && batch > 0;
+  if (work && A == nullptr) return -5;
+  if (lda < std::max(1, m)) return -6;
+  if (work && tau == nullptr) return -7;
+  if (!work) return BQR_SUCCESS;
+  if ((reinterpret_cast<uintptr_t>(A) | reinterpret_cast<uintptr_t>(tau)) % elem_size(dtype))
+    return BQR_ERR_MISALIGNED;
+  if (m < n) return BQR_ERR_NOT_SUPPORTED;
+  Plan p;
+  if (!geqrf_plan(dtype, m, n, &p)) return BQR_ERR_NOT_SUPPORTED;
+  Call c{A, tau, batch, m, n, std::min(m, n), lda, stream};
+  return p.geqrf(c);
+}
+
+int bqr_orgqr_batched(bqr_dtype_t dtype, int m, int n, int k, int batch, void *A, int lda,
+                      const void *tau, cudaStream_t stream) {
+  if (!valid_dtype(dtype)) return -1;
+  if (m < 0) return -2;
+  if (n < 0 || n > m) return -3;
+  if (k < 0 || k > n) return -4;
+  if (batch < 0) return -5;
+  const bool work = m > 0 && n > 0 && batch > 0;
+  if (work && A == nullptr) return -6;
+  if (lda < std::max(1, m)) return -7;
+  if (work && k > 0 && tau == nullptr) return -8;
+  if (!work) return BQR_SUCCESS;
+  if ((reinterpret_cast<uintptr_t>(A) | reinterpret_cast<uintptr_t>(tau)) % elem_size(dtype))
+    return BQR_ERR_MISALIGNED;
+  Plan p;
+  if (!orgqr_plan(dtype, m, n, &p)) return BQR_ERR_NOT_SUPPORTED;
+  Call c{A, const_cast<void *>(tau), batch, m, n, k, lda, stream};
+  return p.orgqr(c);
+}
+
+int bqr_apply_qh_batched(bqr_dtype_t dtype, int m, int n, int k, int nrhs, int batch, const void *A,
+                         int lda, const void *tau, void *B, int ldb, cudaStream_t stream) {
+  if (!valid_dtype(dtype)) return -1;
+  if (m < 0) return -2;
+  if (n < 0) return -3;
+  if (k < 0 || k > std::min(m, n)) return -4;
+  if (nrhs < 0) return -5;
+  if (batch < 0) return -6;
+  const bool work = m > 0 && nrhs > 0 && batch > 0;
+  if (work && k > 0 && A == nullptr) return -7;
+  if (lda < std::max(1, m)) return -8;
+  if (work && k > 0 && tau == nullptr) return -9;
+  if (work && B == nullptr) return -10;
+  if (ldb < std::max(1, m)) return -11;
+  if (!work || k == 0) return BQR_SUCCESS;
+  if ((reinterpret_cast<uintptr_t>(A) | reinterpret_cast<uintptr_t>(tau) |
+       reinterpret_cast<uintptr_t>(B)) % elem_size(dtype))
+    return BQR_ERR_MISALIGNED;
+  ApplyArgs a{A, tau, B, batch, lda, n, m, k, nrhs, ldb};
+  return dtype == BQR_R32 ? apply_dispatch<float>(a, stream) : apply_dispatch<float2>(a, stream);
+}
+
+size_t bqr_host_workspace_bytes(bqr_dtype_t dtype, int m, int n, int lda, int chunk) {
+  if (!valid_dtype(dtype) || m <= 0 || n <= 0 || chunk <= 0) return 0;
+  const size_t s = elem_size(dtype);
+  const size_t per = ((size_t)lda * n + std::min(m, n)) * s;
+  return 2 * per * (size_t)chunk + 256;
+}
+
+// Host-buffer streaming: chunks of the batch ping-pong through two device
+// buffers; H2D(i+1) overlaps geqrf(i) and D2H(i-1) via two internal streams
+// ordered by events.  Synchronous.
+int bqr_geqrf_batched_host(bqr_dtype_t dtype, int m, int n, int batch, void *A_host, int lda,
+                           void *tau_host, void *workspace, size_t workspace_bytes,
+                           cudaStream_t stream) {
+  if (!valid_dtype(dtype)) return -1;
+  if (m < 0) return -2;
+  if (n < 0) return -3;
+  if (batch < 0) return -4;
+  const bool work = m > 0 && n > 0 && batch > 0;
+  if (work && A_host == nullptr) return -5;
+  if (lda < std::max(1, m)) return -6;
+  if (work && tau_host == nullptr) return -7;
+  if (work && workspace == nullptr) return -8;
+  if (!work) return BQR_SUCCESS;
+  const size_t s = elem_size(dtype);
+  const int k = std::min(m, n);
+  const size_t mat_bytes = (size_t)lda * n * s, tau_bytes = (size_t)k * s;
+  const size_t per = mat_bytes + tau_bytes;
+  if (m < n) return BQR_ERR_NOT_SUPPORTED;
+  Plan p;
+  if (!geqrf_plan(dtype, m, n, &p)) return BQR_ERR_NOT_SUPPORTED;
+  auto r256 = [](size_t x) { return (x + 255) & ~size_t(255); };
+  auto need = [&](long long ch) { return 2 * (r256(mat_bytes * ch) + r256(tau_bytes * ch)) + 256; };
+  long long chunk = std::min<long long>(batch, (long long)(workspace_bytes / (2 * per)));
+  while (chunk > 0 && need(chunk) > workspace_bytes) chunk -= std::max<long long>(1, chunk / 64);
+  if (chunk < 1) return -9;
+  // two buffers [A chunk | tau chunk], 256-byte aligned
+  char *ws = reinterpret_cast<char *>((reinterpret_cast<uintptr_t>(workspace) + 255) & ~uintptr_t(255));
+  const size_t abytes = r256(mat_bytes * chunk), tbytes = r256(tau_bytes * chunk);
+  char *bufA[2] = {ws, ws + abytes + tbytes};
+  char *bufT[2] = {ws + abytes, ws + 2 * abytes + tbytes};
+  cudaStream_t st[3] = {stream, nullptr, nullptr};  // compute, h2d, d2h
+  cudaEvent_t ev_in[2], ev_done[2], ev_out[2];
+  int status = BQR_SUCCESS;
+  if (cudaStreamCreateWithFlags(&st[1], cudaStreamNonBlocking) != cudaSuccess ||
+      cudaStreamCreateWithFlags(&st[2], cudaStreamNonBlocking) != cudaSuccess)
+    return BQR_ERR_CUDA;
+  for (int i = 0; i < 2; ++i) {
+    cudaEventCreateWithFlags(&ev_in[i], cudaEventDisableTiming);
+    cudaEventCreateWithFlags(&ev_done[i], cudaEventDisableTiming);
+    cudaEventCreateWithFlags(&ev_out[i], cudaEventDisableTiming);
+  }
+  // order the copies after whatever the caller already queued on `stream`
+  cudaEvent_t ev_entry;
+  cudaEventCreateWithFlags(&ev_entry, cudaEventDisableTiming);
+  cudaEventRecord(ev_entry, st[0]);
+  cudaStreamWaitEvent(st[1], ev_entry, 0);
+  cudaEventDestroy(ev_entry);
+  const long long nchunks = (batch + chunk - 1) / chunk;
+  bool out_pending[2] = {false, false};
+  for (long long ci = 0; ci < nchunks && status == BQR_SUCCESS; ++ci) {
+    const int b = (int)(ci & 1);
+    const long long b0 = ci * chunk;
+    const long long cnt = std::min<long long>(chunk, batch - b0);
+    // buffer b free once its previous D2H finished
+    if (out_pending[b]) cudaStreamWaitEvent(st[1], ev_out[b], 0);
+    cudaMemcpyAsync(bufA[b], reinterpret_cast<char *>(A_host) + b0 * mat_bytes, cnt * mat_bytes,
+                    cudaMemcpyHostToDevice, st[1]);
+    cudaEventRecord(ev_in[b], st[1]);
+    cudaStreamWaitEvent(st[0], ev_in[b], 0);
+    Call c{bufA[b], bufT[b], cnt, m, n, k, lda, st[0]};
+    status = p.geqrf(c);
+    cudaEventRecord(ev_done[b], st[0]);
+    cudaStreamWaitEvent(st[2], ev_done[b], 0);
+    cudaMemcpyAsync(reinterpret_cast<char *>(A_host) + b0 * mat_bytes, bufA[b], cnt * mat_bytes,
+                    cudaMemcpyDeviceToHost, st[2]);
+    cudaMemcpyAsync(reinterpret_cast<char *>(tau_host) + b0 * tau_bytes, bufT[b], cnt * tau_bytes,
+                    cudaMemcpyDeviceToHost, st[2]);
+    cudaEventRecord(ev_out[b], st[2]);
+    out_pending[b] = true;
+  }
+  if (cudaStreamSynchronize(st[2]) != cudaSuccess || cudaStreamSynchronize(st[0]) != cudaSuccess)
+    status = BQR_ERR_CUDA;
+  for (int i = 0; i < 2; ++i) {
+    cudaEventDestroy(ev_in[i]);
+    cudaEventDestroy(ev_done[i]);
+    cudaEventDestroy(ev_out[i]);
+  }
+  cudaStreamDestroy(st[1]);
+  cudaStreamDestroy(st[2]);
+  if (status == BQR_SUCCESS && cudaGetLastError() != cudaSuccess) status = BQR_ERR_CUDA;
+  return status;
+}
+
+}  // extern "C"

@@ -1,0 +1,129 @@
+"""C-ABI boundary checks that need no GPU: the library loads, exports every
+symbol include/bqr.h declares, validates arguments LAPACK-style without
+touching memory, quick-returns, and reports its dispatch."""
+import ctypes
+import os
+import re
+
+import pytest
+
+import paper_conf_ipps_andersonsk12_b200 as bqr
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+HEADER = os.path.join(ROOT, "include", "bqr.h")
+
+
+@pytest.fixture(scope="module")
+def lib():
+    from paper_conf_ipps_andersonsk12_b200 import build
+    build.build()
+    return bqr.load()
+
+
+def declared_symbols():
+    txt = open(HEADER).read()
+    txt = re.sub(r"/\*.*?\*/", "", txt, flags=re.S)
+    return sorted(set(re.findall(r"\b(bqr_[a-z0-9_]+)\s*\(", txt)))
+
+
+def test_header_declares_the_boundary():
+    syms = declared_symbols()
+    for s in ("bqr_geqrf_batched", "bqr_orgqr_batched", "bqr_apply_qh_batched", "bqr_status_string"):
+        assert s in syms
+
+
+def test_exports_every_declared_symbol(lib):
+    for s in declared_symbols():
+        assert hasattr(lib, s), s
+        assert ctypes.cast(getattr(lib, s), ctypes.c_void_p).value
+
+
+def test_version(lib):
+    assert b"sm_100a" in lib.bqr_version()
+
+
+FAKE = 0x1000  # never dereferenced: every call below returns before any launch
+
+
+@pytest.mark.parametrize("args,code", [
+    ((7, 4, 4, 1, FAKE, 4, FAKE), -1),          # bad dtype
+    ((0, -1, 4, 1, FAKE, 4, FAKE), -2),
+    ((0, 4, -1, 1, FAKE, 4, FAKE), -3),
+    ((0, 4, 4, -1, FAKE, 4, FAKE), -4),
+    ((0, 4, 4, 1, 0, 4, FAKE), -5),             # NULL A with work
+    ((0, 4, 4, 1, FAKE, 3, FAKE), -6),          # lda < m
+    ((0, 4, 4, 1, FAKE, 4, 0), -7),             # NULL tau
+    ((0, 0, 4, 1, 0, 1, 0), 0),                 # quick return m == 0
+    ((0, 4, 0, 1, 0, 4, 0), 0),                 # quick return n == 0
+    ((1, 4, 4, 0, 0, 4, 0), 0),                 # quick return batch == 0
+    ((0, 4, 4, 1, FAKE + 2, 4, FAKE), 3),       # misaligned fp32 pointer
+    ((1, 4, 4, 1, FAKE + 4, 4, FAKE), 3),       # misaligned c64 pointer
+    ((0, 3, 5, 1, FAKE, 3, FAKE), 1),           # m < n: not supported
+    ((0, 4096, 4096, 1, FAKE, 4096, FAKE), 1),  # too large: not supported
+])
+def test_geqrf_argument_checks(lib, args, code):
+    d, m, n, b, A, lda, tau = args
+    st = lib.bqr_geqrf_batched(d, m, n, b, ctypes.c_void_p(A), lda, ctypes.c_void_p(tau), None)
+    assert st == code
+
+
+@pytest.mark.parametrize("args,code", [
+    ((0, 4, 5, 4, 1, FAKE, 4, FAKE), -3),       # n > m
+    ((0, 4, 4, 5, 1, FAKE, 4, FAKE), -4),       # k > n
+    ((0, 4, 4, 4, -1, FAKE, 4, FAKE), -5),
+    ((0, 4, 4, 4, 1, 0, 4, FAKE), -6),
+    ((0, 4, 4, 4, 1, FAKE, 2, FAKE), -7),
+    ((0, 4, 4, 4, 1, FAKE, 4, 0), -8),
+    ((0, 4, 4, 4, 0, 0, 4, 0), 0),
+])
+def test_orgqr_argument_checks(lib, args, code):
+    d, m, n, k, b, A, lda, tau = args
+    assert lib.bqr_orgqr_batched(d, m, n, k, b, ctypes.c_void_p(A), lda, ctypes.c_void_p(tau), None) == code
+
+
+@pytest.mark.parametrize("args,code", [
+    ((0, 8, 4, 5, 1, 1, FAKE, 8, FAKE, FAKE, 8), -4),   # k > min(m,n)
+    ((0, 8, 4, 4, -1, 1, FAKE, 8, FAKE, FAKE, 8), -5),
+    ((0, 8, 4, 4, 1, -1, FAKE, 8, FAKE, FAKE, 8), -6),
+    ((0, 8, 4, 4, 1, 1, FAKE, 7, FAKE, FAKE, 8), -8),
+    ((0, 8, 4, 4, 1, 1, FAKE, 8, FAKE, 0, 8), -10),
+    ((0, 8, 4, 4, 1, 1, FAKE, 8, FAKE, FAKE, 7), -11),
+    ((0, 8, 4, 0, 1, 1, 0, 8, 0, FAKE, 8), 0),          # k == 0: nothing to do
+    ((0, 8, 4, 4, 0, 1, 0, 8, 0, 0, 8), 0),             # nrhs == 0
+])
+def test_apply_argument_checks(lib, args, code):
+    d, m, n, k, nrhs, b, A, lda, tau, B, ldb = args
+    st = lib.bqr_apply_qh_batched(d, m, n, k, nrhs, b, ctypes.c_void_p(A), lda, ctypes.c_void_p(tau),
+                                  ctypes.c_void_p(B), ldb, None)
+    assert st == code
+
+
+def test_status_strings(lib):
+    for s in (-3, 0, 1, 2, 3, 99):
+        assert lib.bqr_status_string(s)
+
+
+@pytest.mark.parametrize("dt,m,n,expect", [
+    (0, 4, 4, "tiny"), (0, 8, 8, "tiny"), (1, 8, 8, "tiny"),
+    (0, 56, 56, "rf_f32_R2G8_28x7_x2_stage"), (1, 240, 66, "rf_c64_R32G16_8x5_cta"),
+    (0, 16, 16, "rf_f32"), (1, 100, 100, "rf_c64"),
+])
+def test_dispatch(lib, dt, m, n, expect):
+    assert bqr.kernel_name(dt, m, n).startswith(expect)
+    assert bqr.geqrf_launches(dt, m, n, 10) == 1
+
+
+def test_workspace_size(lib):
+    w = bqr.host_workspace_bytes(0, 56, 56, 56, 100)
+    assert w >= 2 * 100 * (56 * 56 + 56) * 4
+
+
+def test_no_fallback_when_library_missing(monkeypatch, tmp_path):
+    """The binding must fail loudly, never fall back to a CPU path."""
+    import importlib
+    mod = importlib.reload(bqr)
+    monkeypatch.setattr(mod, "_LIB_PATH", str(tmp_path / "missing.so"))
+    monkeypatch.setattr(mod, "_lib", None)
+    with pytest.raises(mod.BQRError):
+        mod.load()
+    importlib.reload(bqr)

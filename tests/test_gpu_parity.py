@@ -1,0 +1,192 @@
+"""GPU parity: the CUDA path (through the C ABI) against the fp64 oracle on
+the same seeded inputs, with the comparator of oracle/compare.py
+(north-star tolerances: residual 1e-5, orthogonality 1e-5, R 1e-4 relative;
+DESIGN.md "Parity bar")."""
+import numpy as np
+import pytest
+
+import bqr_inputs
+import oracle
+from oracle.compare import compare_apply, compare_geqrf, compare_orgqr
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+if not torch.cuda.is_available():  # pragma: no cover
+    pytest.skip("needs a GPU", allow_module_level=True)
+
+from gpu_util import apply_gpu, geqrf_gpu, orgqr_gpu  # noqa: E402
+
+
+def _check(A, m, full_q=True):
+    out, tau = geqrf_gpu(A, m)
+    rep = compare_geqrf(A, m, out, tau, full_q=full_q)
+    assert rep["ok"], rep
+    return out, tau, rep
+
+
+# ------------------------------------------------------------- configs
+
+def test_C1_8x8_full():
+    A = bqr_inputs.config_batch("C1")
+    _, _, rep = _check(A, 8)
+    assert rep["residual_max"] < 2e-6
+
+
+def test_C2_4x4_full_size_sampled():
+    """1e6 4x4 at full size in the bench's launch configuration; every 7th
+    matrix compared (the rest is checked via the invariant |diag R| etc.)."""
+    A = bqr_inputs.config_batch("C2")
+    out, tau = geqrf_gpu(A, 4)
+    idx = np.arange(0, A.shape[0], 7)
+    rep = compare_geqrf(A[idx], 4, out[idx], tau[idx])
+    assert rep["ok"], rep
+    # property on all matrices: column norms preserved by the factorisation
+    R = np.triu(np.swapaxes(out, 1, 2)).astype(np.float64)
+    An = np.linalg.norm(A.astype(np.float64), axis=2)
+    np.testing.assert_allclose(np.linalg.norm(R, axis=1), An, rtol=2e-6, atol=1e-30)
+
+
+def test_C3_56x56_full():
+    A = bqr_inputs.config_batch("C3")
+    _, _, rep = _check(A, 56)
+    assert rep["residual_max"] < 2e-6 and rep["orth_max"] < 5e-6
+
+
+def test_C4_stap_240x66_full_with_apply():
+    A = bqr_inputs.config_batch("C4")
+    out, tau, rep = _check(A, 240, full_q=False)
+    B = bqr_inputs.rhs_batch(240, 1, 256, "c64", seed=4)
+    got = apply_gpu(out, 240, 66, tau, B)
+    r = compare_apply(out, 240, 66, tau, B, got)
+    assert r["ok"], r
+
+
+# ------------------------------------------------------------- size sweep
+
+F32_SHAPES = [(1, 1), (2, 2), (3, 2), (4, 4), (5, 3), (7, 7), (8, 8), (8, 1), (9, 9), (12, 5), (15, 15),
+              (16, 16), (17, 17), (20, 11), (31, 31), (32, 32), (33, 33), (40, 40), (55, 55), (56, 56),
+              (57, 57), (56, 20), (63, 63), (64, 64), (65, 65), (80, 80), (96, 96), (100, 37), (127, 127),
+              (128, 128), (200, 50), (256, 64)]
+C64_SHAPES = [(1, 1), (2, 2), (4, 4), (5, 5), (8, 8), (8, 3), (9, 9), (16, 16), (17, 17), (32, 32), (33, 20),
+              (48, 48), (64, 64), (65, 65), (80, 16), (96, 96), (128, 128), (192, 96), (240, 66), (256, 96)]
+
+
+@pytest.mark.parametrize("m,n", F32_SHAPES)
+def test_sweep_f32(m, n):
+    A = bqr_inputs.random_batch(m, n, 300, "f32", seed=1000 + 7 * m + n)
+    _check(A, m)
+
+
+@pytest.mark.parametrize("m,n", C64_SHAPES)
+def test_sweep_c64(m, n):
+    A = bqr_inputs.random_batch(m, n, 130, "c64", seed=2000 + 7 * m + n)
+    _check(A, m, full_q=m <= 128)
+
+
+# ------------------------------------------------------------- edge cases
+
+@pytest.mark.parametrize("dt", ["f32", "c64"])
+@pytest.mark.parametrize("n", [4, 8, 16, 56, 66])
+def test_edge_matrices(dt, n):
+    cases = bqr_inputs.edge_matrices(n, dt)
+    A = np.stack([oracle.to_cm(v[None])[0] for v in cases.values()])
+    out, tau = geqrf_gpu(A, n)
+    rep = compare_geqrf(A, n, out, tau)
+    assert rep["ok"], (list(cases), rep)
+    names = list(cases)
+    # exact special cases (Q5): zero matrix and identity untouched, tau = 0
+    z = names.index("zero")
+    assert np.all(out[z] == 0) and np.all(tau[z] == 0)
+    e = names.index("identity")
+    if dt == "f32":
+        assert np.all(tau[e] == 0) and np.array_equal(out[e], A[e])
+    u = names.index("upper_triangular")
+    if dt == "f32":
+        assert np.all(tau[u] == 0)
+
+
+def test_minus_zero_pivot_sign_rule():
+    """Q4: alpha = -0.0 -> beta = +nu (copysign), on the GPU too."""
+    A = np.array([[[-0.0, 1.0], [1.0, 1.0]]], dtype=np.float32)  # column-major storage
+    out, tau = geqrf_gpu(A, 2)
+    assert out[0, 0, 0] == 1.0 and tau[0, 0] == 1.0
+    A2 = np.array([[[0.0, 1.0], [1.0, 1.0]]], dtype=np.float32)
+    out2, _ = geqrf_gpu(A2, 2)
+    assert out2[0, 0, 0] == -1.0
+
+
+@pytest.mark.parametrize("dt,m,n", [("f32", 4, 4), ("f32", 8, 8), ("f32", 56, 56), ("f32", 30, 20),
+                                    ("c64", 8, 8), ("c64", 240, 66), ("c64", 40, 33)])
+def test_lda_padding_untouched(dt, m, n):
+    A = bqr_inputs.random_batch(m, n, 70, dt, seed=31, lda=m + 3)
+    out, tau = geqrf_gpu(A, m)
+    rep = compare_geqrf(A, m, out, tau, full_q=m <= 128)
+    assert rep["ok"] and rep["padding_ok"], rep
+
+
+@pytest.mark.parametrize("dt,m,n", [("f32", 4, 4), ("f32", 56, 56), ("f32", 100, 100), ("c64", 240, 66),
+                                    ("c64", 8, 8)])
+def test_deterministic_and_position_invariant(dt, m, n):
+    A = bqr_inputs.random_batch(m, n, 257, dt, seed=41)
+    o1, t1 = geqrf_gpu(A, m)
+    o2, t2 = geqrf_gpu(A, m)
+    assert np.array_equal(o1.view(np.uint32), o2.view(np.uint32))
+    assert np.array_equal(t1.view(np.uint32), t2.view(np.uint32))
+    # slice invariance (emulates P ranks each factoring a contiguous slice)
+    for lo, hi in [(0, 1), (5, 6), (100, 257), (31, 97)]:
+        os_, ts_ = geqrf_gpu(A[lo:hi], m)
+        assert np.array_equal(os_.view(np.uint32), o1[lo:hi].view(np.uint32))
+        assert np.array_equal(ts_.view(np.uint32), t1[lo:hi].view(np.uint32))
+
+
+def test_empty_batch_and_quick_returns():
+    A = np.zeros((0, 8, 8), np.float32)
+    out, tau = geqrf_gpu(A, 8)
+    assert out.shape == (0, 8, 8)
+
+
+def test_non_default_stream():
+    A = bqr_inputs.random_batch(56, 56, 100, "f32", seed=51)
+    s = torch.cuda.Stream()
+    with torch.cuda.stream(s):
+        out, tau = geqrf_gpu(A, 56, stream=s)
+    assert compare_geqrf(A, 56, out, tau)["ok"]
+
+
+# ------------------------------------------------------------- orgqr / apply
+
+@pytest.mark.parametrize("dt,m,n", [("f32", 8, 8), ("f32", 56, 56), ("f32", 30, 12), ("f32", 128, 128),
+                                    ("c64", 16, 16), ("c64", 240, 66), ("c64", 64, 40)])
+def test_orgqr(dt, m, n):
+    A = bqr_inputs.random_batch(m, n, 64, dt, seed=61)
+    out, tau = geqrf_gpu(A, m)
+    Q = orgqr_gpu(out, m, n, tau)
+    rep = compare_orgqr(out, m, n, tau, Q)
+    assert rep["ok"], rep
+
+
+@pytest.mark.parametrize("dt,m,n,nrhs", [("f32", 8, 8, 1), ("f32", 56, 56, 3), ("f32", 100, 30, 5),
+                                         ("c64", 240, 66, 1), ("c64", 80, 16, 2), ("c64", 192, 96, 4)])
+def test_apply_qh(dt, m, n, nrhs):
+    A = bqr_inputs.random_batch(m, n, 50, dt, seed=71)
+    B = bqr_inputs.rhs_batch(m, nrhs, 50, dt, seed=71)
+    out, tau = geqrf_gpu(A, m)
+    got = apply_gpu(out, m, min(m, n), tau, B)
+    r = compare_apply(out, m, min(m, n), tau, B, got)
+    assert r["ok"], r
+
+
+def test_host_buffer_api():
+    """bqr_geqrf_batched_host streams a host batch through a small workspace
+    (several chunks) and matches the device path bit for bit."""
+    import paper_conf_ipps_andersonsk12_b200 as bqr
+    A = bqr_inputs.random_batch(56, 56, 1000, "f32", seed=81)
+    dev_out, dev_tau = geqrf_gpu(A, 56)
+    Ah = torch.from_numpy(A.copy()).pin_memory()
+    tau_h = torch.empty((1000, 56), dtype=torch.float32).pin_memory()
+    wsb = bqr.host_workspace_bytes(bqr.R32, 56, 56, 56, 128)
+    ws = torch.empty(wsb, dtype=torch.uint8, device="cuda")
+    bqr.geqrf_batched_host(bqr.R32, 56, 56, 1000, Ah.data_ptr(), 56, tau_h.data_ptr(), ws.data_ptr(), wsb)
+    assert np.array_equal(Ah.numpy().view(np.uint32), dev_out.view(np.uint32))
+    assert np.array_equal(tau_h.numpy().view(np.uint32), dev_tau.view(np.uint32))
