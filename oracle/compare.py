@@ -88,13 +88,16 @@ def compare_geqrf(A_cm: np.ndarray, m: int, out_cm: np.ndarray, tau_gpu: np.ndar
     d = np.sign(dg) * np.sign(dr)
     d = np.where(d == 0, 1.0, d)
     flips = d < 0
-    bad_flip = flips & (margin[:, :k] >= FLIP_MARGIN)
+    # numerical rank: rows before the first negligible reference pivot.  Past
+    # it the reflectors are formed from rounding noise (reading Q5), so only
+    # the residual and orthogonality bind there -- sign flips included.
+    tiny = np.abs(dr) <= 1e-4 * np.where(zero, 1.0, normA)[:, None]
+    first_tiny = np.where(tiny.any(axis=1), tiny.argmax(axis=1), k)
+    below_rank = np.arange(k)[None, :] < first_tiny[:, None]
+    bad_flip = flips & (margin[:, :k] >= FLIP_MARGIN) & below_rank
     rep["flips"] = int(flips.sum())
     rep["bad_flips"] = int(bad_flip.sum())
     colnorm = np.linalg.norm(A, axis=1)  # (batch, n): ||A e_j||
-    # numerical rank: rows before the first negligible reference pivot
-    tiny = np.abs(dr) <= 1e-4 * np.where(zero, 1.0, normA)[:, None]
-    first_tiny = np.where(tiny.any(axis=1), tiny.argmax(axis=1), k)
     rowmask = np.arange(m)[None, :] < first_tiny[:, None]
     Rg_s = Rg * np.concatenate([d, np.ones((batch, m - k))], axis=1)[:, :, None] if m > k else Rg * d[:, :, None]
     scale = np.maximum(np.abs(Rr), colnorm[:, None, :])
