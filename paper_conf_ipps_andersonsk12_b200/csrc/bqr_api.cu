@@ -12,6 +12,7 @@
 #include <atomic>
 #include <cstdint>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <mutex>
 
@@ -121,28 +122,54 @@ int launch_tiny(const Call &c) {
   }
 
 struct ClassEntry {
-  int mmax, nmax;  // class bounds
-  int exact_m, exact_n;
+  bqr_dtype_t dt;
+  int mmax, nmax;           // class bounds (m <= mmax, n <= nmax)
+  int exact_m, exact_n;     // > 0: preferred for exactly this shape
+  bool alt;                 // alternative variant: only via BQR_FORCE_VARIANT
   Plan plan;
 };
 
-const ClassEntry kF32[] = {
-    {56, 56, 56, 56, RF_PLAN(float, 2, 8, 28, 7, 2, true, "rf_f32_R2G8_28x7_x2_stage")},
-    {16, 16, 0, 0, RF_PLAN(float, 2, 4, 8, 4, 8, true, "rf_f32_R2G4_8x4_x8_stage")},
-    {32, 32, 0, 0, RF_PLAN(float, 2, 8, 16, 4, 4, true, "rf_f32_R2G8_16x4_x4_stage")},
-    {64, 64, 0, 0, RF_PLAN(float, 4, 8, 16, 8, 2, true, "rf_f32_R4G8_16x8_x2_stage")},
-    {128, 128, 0, 0, RF_PLAN(float, 32, 8, 4, 16, 1, false, "rf_f32_R32G8_4x16_cta")},
-    {256, 64, 0, 0, RF_PLAN(float, 32, 8, 8, 8, 1, false, "rf_f32_R32G8_8x8_cta")},
+// Size classes.  Order matters: exact shapes first,
+// then the smallest class that holds (m, n).
+const ClassEntry kClasses[] = {
+    // headline shapes, exact fits
+    {BQR_R32, 56, 56, 56, 56, false, RF_PLAN(float, 2, 8, 28, 7, 2, true, "rf_f32_R2G8_28x7_x2_stage")},
+    {BQR_C64, 240, 66, 240, 66, false, RF_PLAN(float2, 16, 22, 15, 3, 1, false, "rf_c64_R16G22_15x3_cta")},
+    // alternatives kept for measurement (BQR_FORCE_VARIANT)
+    {BQR_R32, 56, 56, 56, 56, true, RF_PLAN(float, 4, 8, 14, 7, 1, true, "rf_f32_R4G8_14x7_x1_stage")},
+    {BQR_R32, 56, 56, 56, 56, true, RF_PLAN(float, 4, 4, 14, 14, 2, true, "rf_f32_R4G4_14x14_x2_stage")},
+    {BQR_C64, 240, 66, 240, 66, true, RF_PLAN(float2, 32, 16, 8, 5, 1, false, "rf_c64_R32G16_8x5_cta")},
+    {BQR_C64, 256, 66, 240, 66, true, RF_PLAN(float2, 32, 11, 8, 6, 1, false, "rf_c64_R32G11_8x6_cta")},
+    // fp32 classes
+    {BQR_R32, 16, 16, 0, 0, false, RF_PLAN(float, 2, 4, 8, 4, 8, true, "rf_f32_R2G4_8x4_x8_stage")},
+    {BQR_R32, 32, 32, 0, 0, false, RF_PLAN(float, 2, 8, 16, 4, 4, true, "rf_f32_R2G8_16x4_x4_stage")},
+    {BQR_R32, 64, 64, 0, 0, false, RF_PLAN(float, 4, 8, 16, 8, 2, true, "rf_f32_R4G8_16x8_x2_stage")},
+    {BQR_R32, 128, 128, 0, 0, false, RF_PLAN(float, 32, 8, 4, 16, 1, false, "rf_f32_R32G8_4x16_cta")},
+    {BQR_R32, 256, 64, 0, 0, false, RF_PLAN(float, 32, 8, 8, 8, 1, false, "rf_f32_R32G8_8x8_cta")},
+    // complex64 classes
+    {BQR_C64, 16, 16, 0, 0, false, RF_PLAN(float2, 8, 4, 2, 4, 1, false, "rf_c64_R8G4_2x4_warp")},
+    {BQR_C64, 32, 32, 0, 0, false, RF_PLAN(float2, 8, 4, 4, 8, 1, false, "rf_c64_R8G4_4x8_warp")},
+    {BQR_C64, 64, 64, 0, 0, false, RF_PLAN(float2, 16, 8, 4, 8, 1, false, "rf_c64_R16G8_4x8_cta")},
+    {BQR_C64, 128, 128, 0, 0, false, RF_PLAN(float2, 32, 16, 4, 8, 1, false, "rf_c64_R32G16_4x8_cta")},
+    {BQR_C64, 256, 96, 0, 0, false, RF_PLAN(float2, 32, 16, 8, 6, 1, false, "rf_c64_R32G16_8x6_cta")},
 };
 
-const ClassEntry kC64[] = {
-    {240, 66, 240, 66, RF_PLAN(float2, 32, 16, 8, 5, 1, false, "rf_c64_R32G16_8x5_cta")},
-    {16, 16, 0, 0, RF_PLAN(float2, 8, 4, 2, 4, 1, false, "rf_c64_R8G4_2x4_warp")},
-    {32, 32, 0, 0, RF_PLAN(float2, 8, 4, 4, 8, 1, false, "rf_c64_R8G4_4x8_warp")},
-    {64, 64, 0, 0, RF_PLAN(float2, 16, 8, 4, 8, 1, false, "rf_c64_R16G8_4x8_cta")},
-    {128, 128, 0, 0, RF_PLAN(float2, 32, 16, 4, 8, 1, false, "rf_c64_R32G16_4x8_cta")},
-    {256, 96, 0, 0, RF_PLAN(float2, 32, 16, 8, 6, 1, false, "rf_c64_R32G16_8x6_cta")},
-};
+const char *forced_variant() {
+  static const char *v = std::getenv("BQR_FORCE_VARIANT");
+  return (v && *v) ? v : nullptr;
+}
+
+const Plan *pick(bqr_dtype_t dt, int m, int n) {
+  if (const char *f = forced_variant()) {
+    for (const auto &e : kClasses)
+      if (e.dt == dt && std::strcmp(e.plan.name, f) == 0 && m <= e.mmax && n <= e.nmax) return &e.plan;
+  }
+  for (const auto &e : kClasses)
+    if (e.dt == dt && !e.alt && e.exact_m == m && e.exact_n == n) return &e.plan;
+  for (const auto &e : kClasses)
+    if (e.dt == dt && !e.alt && e.exact_m == 0 && m <= e.mmax && n <= e.nmax) return &e.plan;
+  return nullptr;
+}
 
 // tiny exact sizes 1 <= n <= m <= 8
 template <class T, int M>
@@ -172,22 +199,13 @@ Plan tiny_plan(int m, int n) {
   return Plan{nullptr, nullptr, nullptr};
 }
 
-template <size_t N>
-const Plan *pick(const ClassEntry (&tab)[N], int m, int n) {
-  for (const auto &e : tab)
-    if (e.exact_m == m && e.exact_n == n) return &e.plan;
-  for (const auto &e : tab)
-    if (e.exact_m == 0 && m <= e.mmax && n <= e.nmax) return &e.plan;
-  return nullptr;
-}
-
 // geqrf plan; tiny sizes get their own thread-per-matrix kernel.
 bool geqrf_plan(bqr_dtype_t dt, int m, int n, Plan *out) {
-  if (m <= 8 && n <= m) {
+  if (m <= 8 && n <= m && !forced_variant()) {
     *out = dt == BQR_R32 ? tiny_plan<float>(m, n) : tiny_plan<float2>(m, n);
     return out->geqrf != nullptr;
   }
-  const Plan *p = dt == BQR_R32 ? pick(kF32, m, n) : pick(kC64, m, n);
+  const Plan *p = pick(dt, m, n);
   if (!p) return false;
   *out = *p;
   return true;
@@ -195,7 +213,7 @@ bool geqrf_plan(bqr_dtype_t dt, int m, int n, Plan *out) {
 
 // orgqr has no thread-per-matrix kernel: tiny shapes use the smallest rf class
 bool orgqr_plan(bqr_dtype_t dt, int m, int n, Plan *out) {
-  const Plan *p = dt == BQR_R32 ? pick(kF32, m, n) : pick(kC64, m, n);
+  const Plan *p = pick(dt, m, n);
   if (!p) return false;
   *out = *p;
   return true;
@@ -220,6 +238,34 @@ int apply_dispatch(const ApplyArgs &a, cudaStream_t s) {
   if (mr <= 4) return launch_apply<T, 4, 2>(a, s);
   if (mr <= 8) return launch_apply<T, 8, 1>(a, s);
   return BQR_ERR_NOT_SUPPORTED;
+}
+
+// self-test of the branch-free IEEE helpers (bqr_common.cuh) against the
+// CUDA library's sqrt.rn / div.rn on random normal operands spanning the
+// exponent range the contract (reading Q6) can produce.
+__device__ __forceinline__ unsigned hash32(unsigned x) {
+  x ^= x >> 16; x *= 0x7feb352dU; x ^= x >> 15; x *= 0x846ca68bU; x ^= x >> 16;
+  return x;
+}
+__device__ __forceinline__ float rand_normal_float(unsigned h, int emin, int emax) {
+  const unsigned mant = h & 0x7fffffU;
+  const int e = emin + (int)((h >> 23) % (unsigned)(emax - emin + 1));
+  return __uint_as_float(((unsigned)(e + 127) << 23) | mant);
+}
+__global__ void selftest_math_kernel(long long n, unsigned seed, unsigned long long *counts) {
+  unsigned long long bad_sqrt = 0, bad_div = 0, bad_rcp = 0;
+  for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x) {
+    const unsigned h1 = hash32((unsigned)i * 2654435761U ^ seed), h2 = hash32(h1 ^ 0x9e3779b9U);
+    const float x = rand_normal_float(h1, -100, 100);           // sigma / |z|^2 range
+    const float a = rand_normal_float(h2, -50, 50) * ((h2 & 1) ? -1.f : 1.f);
+    const float b = rand_normal_float(h1 ^ h2, -50, 50) * ((h1 & 2) ? -1.f : 1.f);
+    bad_sqrt += __float_as_uint(bqr::sqrt_rn(x)) != __float_as_uint(__fsqrt_rn(x));
+    bad_div += __float_as_uint(bqr::div_rn(a, b)) != __float_as_uint(__fdiv_rn(a, b));
+    bad_rcp += __float_as_uint(bqr::div_rn(1.0f, b)) != __float_as_uint(__frcp_rn(b));
+  }
+  atomicAdd(&counts[0], bad_sqrt);
+  atomicAdd(&counts[1], bad_div);
+  atomicAdd(&counts[2], bad_rcp);
 }
 
 bool valid_dtype(int d) { return d == BQR_R32 || d == BQR_C64; }
@@ -315,6 +361,13 @@ int bqr_apply_qh_batched(bqr_dtype_t dtype, int m, int n, int k, int nrhs, int b
     return BQR_ERR_MISALIGNED;
   ApplyArgs a{A, tau, B, batch, lda, n, m, k, nrhs, ldb};
   return dtype == BQR_R32 ? apply_dispatch<float>(a, stream) : apply_dispatch<float2>(a, stream);
+}
+
+int bqr_selftest_math(long long n, unsigned seed, unsigned long long *counts, cudaStream_t stream) {
+  if (n < 0) return -1;
+  if (counts == nullptr) return -3;
+  selftest_math_kernel<<<1184, 256, 0, stream>>>(n, seed, counts);
+  return finish_launch();
 }
 
 size_t bqr_host_workspace_bytes(bqr_dtype_t dtype, int m, int n, int lda, int chunk) {

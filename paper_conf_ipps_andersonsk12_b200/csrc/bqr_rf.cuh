@@ -10,21 +10,26 @@
 // B200 re-design (not a port):
 //   * a "group" of R x G threads owns one matrix; rows are cyclic over the R
 //     lanes of a warp segment (so every column reduction -- the norm and the
-//     matrix-vector product -- is a warp shuffle butterfly, no barrier, no
+//     matrix-vector product -- is a warp-shuffle butterfly, no barrier, no
 //     thread-0 serial loop) and columns are cyclic over the G column groups;
 //     R and G need not be equal (the paper needed p = sqrt(p)^2);
 //   * a group is a sub-warp (several matrices per warp, e.g. 2 x 56x56 fp32
-//     per warp), a warp, or a CTA (e.g. 240x66 c64 across 16 warps);
-//   * the reflector is computed redundantly by every lane of the owning
-//     column group with IEEE sqrt/div (north star; not the 22-bit hardware
-//     path of P:L321); its vector is published through a double-buffered
+//     per warp), a warp, or a CTA (e.g. 240x66 c64 over 11 warps);
+//   * look-ahead: inside step k the column group that owns column k+1 first
+//     applies H_k to that column, forms reflector k+1 (norm, IEEE sqrt/div)
+//     and only then applies H_k to its other columns, so the serial
+//     reflector chain overlaps independent FMAs instead of idling the SM;
+//     the new vector is published into the other half of a double-buffered
 //     shared-memory slot, so ONE group barrier per column suffices;
 //   * the compile-time panel recursion advances the first live
 //     register row/column slot per panel, so finished rows/columns cost
 //     nothing; inside a panel the column loop is a runtime loop (small code);
+//   * Householder vectors live in shared memory row-lane-major, so every
+//     lane re-reads its rows with 16-byte loads instead of holding them in
+//     registers (the matrix itself needs the register file);
 //   * global <-> register staging either directly (row lanes >= 8: each warp
-//     access is a contiguous column segment) or through a bank-conflict-free
-//     padded shared-memory tile filled by 16-byte cp.async (small R).
+//     access is a contiguous column segment) or through a shared-memory tile
+//     filled by 16-byte cp.async (small R).
 #pragma once
 #include "bqr_common.cuh"
 
@@ -47,7 +52,27 @@ __device__ __forceinline__ void group_sync(int grp) {
   } else if constexpr (GPB == 1) {
     __syncthreads();
   } else {
-    asm volatile("bar.sync %0, %1;" ::"r"(1 + grp), "r"(GT) : "memory");
+    asm volatile("bar.sync %0, %1;" ::"r"(8 + grp), "r"(GT) : "memory");
+  }
+}
+
+// Producer/consumer step barrier of a multi-warp group: the warp that
+// publishes reflector k arrives (release, no wait) on named barrier
+// 1 + k % NB; every other warp syncs on it before reading the vector.  A
+// warp can run ahead only through the steps whose columns it owns itself
+// (at most 32/R in a row), so NB = 32/R + 2 rotating IDs (and as many vector
+// buffers) keep an early arrival off an instance that has not completed.
+template <int GT, int NB>
+__device__ __forceinline__ void step_arrive(int k) {
+  __syncwarp();
+  if constexpr (GT > 32) asm volatile("bar.arrive %0, %1;" ::"r"(1 + k % NB), "r"(GT) : "memory");
+}
+template <int GT, int NB>
+__device__ __forceinline__ void step_wait(int k) {
+  if constexpr (GT <= 32) {
+    __syncwarp();
+  } else {
+    asm volatile("bar.sync %0, %1;" ::"r"(1 + k % NB), "r"(GT) : "memory");
   }
 }
 
@@ -55,8 +80,28 @@ __device__ __forceinline__ void cp_async16(void *smem_dst, const void *gmem_src)
   unsigned s = (unsigned)__cvta_generic_to_shared(smem_dst);
   asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(s), "l"(gmem_src) : "memory");
 }
-__device__ __forceinline__ void cp_async_wait_all() {
-  asm volatile("cp.async.wait_all;\n" ::: "memory");
+__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;\n" ::: "memory"); }
+
+// 16-byte shared loads that the compiler may not merge across passes (keeps
+// the Householder vector out of the register file between the
+// matrix-vector product and the rank-1 update).
+__device__ __forceinline__ float4 lds128(const void *p) {
+  float4 v;
+  unsigned s = (unsigned)__cvta_generic_to_shared(p);
+  asm volatile("ld.shared.v4.f32 {%0,%1,%2,%3}, [%4];" : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "r"(s));
+  return v;
+}
+__device__ __forceinline__ float lds32(const void *p) {
+  float v;
+  unsigned s = (unsigned)__cvta_generic_to_shared(p);
+  asm volatile("ld.shared.f32 %0, [%1];" : "=f"(v) : "r"(s));
+  return v;
+}
+__device__ __forceinline__ float2 lds64(const void *p) {
+  float2 v;
+  unsigned s = (unsigned)__cvta_generic_to_shared(p);
+  asm volatile("ld.shared.v2.f32 {%0,%1}, [%2];" : "=f"(v.x), "=f"(v.y) : "r"(s));
+  return v;
 }
 
 template <class T, int R, int G, int MR, int NC, int GPB, bool STAGE>
@@ -65,14 +110,27 @@ struct RfCfg {
   static constexpr int NT = GT * GPB;
   static constexpr int MMAX = R * MR;
   static constexpr int NMAX = G * NC;
-  static constexpr int E = sizeof(T) / 4;
-  // per-group small smem: double-buffered Householder vector + tau list
-  static constexpr int kSmallWords = (2 * MMAX + NMAX) * E;
+  static constexpr int E = sizeof(T) / 4;     // 32-bit words per element
+  static constexpr int VW = 4 / E;            // elements per 16-byte vector
+  // row-lane-major vector buffer: rows of lane rg at [rg*MRP, rg*MRP+MR);
+  // MRP*E == 4 (mod 32) spreads the R lanes over distinct bank quads.
+  static constexpr int mrp_calc() {
+    int x = ((MR + VW - 1) / VW) * VW;
+    if (R == 1) return x;
+    while ((x * E) % 32 != 4) x += VW;
+    return x;
+  }
+  static constexpr int MRP = mrp_calc();
+  static constexpr int VB = R * MRP;          // elements per vector buffer
+  // multi-warp groups publish ahead without a full barrier (see step_arrive)
+  static constexpr int NBUF = GT <= 32 ? 2 : 32 / R + 2;
+  static_assert(GT <= 32 || GPB == 1, "multi-warp groups: one group per CTA");
+  static constexpr int kSmallWords = ((NBUF * VB + NMAX) * E + 3) / 4 * 4;
   static constexpr int kSmallAll = ((GPB * kSmallWords + 31) / 32) * 32;
   static_assert(R >= 1 && R <= 32 && (R & (R - 1)) == 0, "R must be a power of two <= 32");
-  static_assert(GT <= 32 ? (32 % GT == 0) : (GT % 32 == 0), "group must tile warps");
+  static_assert(GT <= 32 ? (32 % GT == 0) : (GT % 32 == 0 && 32 % R == 0), "group must tile warps");
   static_assert(!STAGE || E == 1, "smem staging implemented for fp32");
-  // rows that may equal the pivot row inside one panel (see column())
+  // register rows that may hold the pivot row of a column inside one panel
   static constexpr int NMASK = (G + R - 1) / R + 1;
 };
 
@@ -81,86 +139,224 @@ struct RfKernel {
   using Cfg = RfCfg<T, R, G, MR, NC, GPB, STAGE>;
   using X = El<T>;
   static constexpr int GT = Cfg::GT;
-  static constexpr int MMAX = Cfg::MMAX;
+  static constexpr int VW = Cfg::VW;
+  static constexpr int MRP = Cfg::MRP;
+  static constexpr int VB = Cfg::VB;
+  static constexpr int NBUF = Cfg::NBUF;
+  static __device__ __forceinline__ int buf(int k) { return k % NBUF; }
 
   struct Ctx {
-    T *vbuf;   // [2][MMAX]
+    T *vbuf;   // [NBUF][VB]
     T *taus;   // [NMAX]
     int rg, cg, t, lane, grp;
     int kmax;
   };
 
-  // One Householder step on column k (panel P, first live register row I0).
-  template <int P, int I0>
-  static __device__ __forceinline__ void column(Ctx &c, T (&a)[MR][NC], int k) {
-    const int kk = k - P * G;  // owning column group
-    T *vb = c.vbuf + (k & 1) * MMAX;
-    // ---- reflector (xLARFG) on the owning column group: Table VI "Column"
-    bool warp_has_owner;
-    if constexpr (GT <= 32) {
-      warp_has_owner = true;
-    } else {
-      warp_has_owner = (kk / (32 / R)) == (c.t >> 5);
-    }
-    if (warp_has_owner) {
-      float sig = 0.f;
-      T alpha = X::zero();
+  struct Look {
+    T scal, tau;
+    float beta;
+  };
+
+  // ------------------------------------------------------------ smem vector I/O
+  // load rows [I0, MR) of this lane's Householder vector (others left unset)
+  template <int I0>
+  static __device__ __forceinline__ void load_v(const T *base, T (&v)[MR]) {
 #pragma unroll
-      for (int i = I0; i < MR; ++i) {
-        const int r = c.rg + R * i;
-        const T x = a[i][P];
-        if (i < I0 + Cfg::NMASK) {
-          sig = X::abs2_acc(X::sel(r > k, x, X::zero()), sig);
-          alpha = X::sel(r == k, x, alpha);
+    for (int q = 0; q < MR; ++q) {
+      if (q < I0) continue;
+      const int q0 = q - q % VW;
+      const bool vec_start = (q % VW == 0) && (q + VW <= MR);
+      const bool in_vec = (q % VW != 0) && (q0 >= I0) && (q0 + VW <= MR);
+      if (vec_start) {
+        const float4 f = lds128(base + q);
+        if constexpr (VW == 4) {
+          v[q] = X::make(f.x, 0.f);
+          v[q + 1 < MR ? q + 1 : q] = X::make(f.y, 0.f);
+          v[q + 2 < MR ? q + 2 : q] = X::make(f.z, 0.f);
+          v[q + 3 < MR ? q + 3 : q] = X::make(f.w, 0.f);
         } else {
-          sig = X::abs2_acc(x, sig);
+          set_word(v[q], 0, f.x);
+          set_word(v[q], 1, f.y);
+          set_word(v[q + 1 < MR ? q + 1 : q], 0, f.z);
+          set_word(v[q + 1 < MR ? q + 1 : q], 1, f.w);
         }
-      }
-      sig = row_allreduce_f<R>(sig);
-      if constexpr (R > 1) alpha = X::shfl(alpha, (c.lane & ~(R - 1)) | (k & (R - 1)));
-      const Reflector<T> h = make_reflector(alpha, sig);
-      if (c.cg == kk) {
-        // scale x, write beta, publish v (v_k = 1, v_r = 0 above the pivot)
-#pragma unroll
-        for (int i = I0; i < MR; ++i) {
-          const int r = c.rg + R * i;
-          T x = a[i][P];
-          T v;
-          if (i < I0 + Cfg::NMASK) {
-            const T xs = X::mul(x, h.scal);
-            v = X::sel(r > k, xs, X::sel(r == k, X::one(), X::zero()));
-            x = X::sel(r > k, xs, X::sel(r == k, X::make(h.beta, 0.f), x));
-          } else {
-            v = X::mul(x, h.scal);
-            x = v;
-          }
-          a[i][P] = x;
-          vb[r] = v;
+      } else if (!in_vec) {
+        if constexpr (VW == 4) {
+          v[q] = X::make(lds32(base + q), 0.f);
+        } else {
+          const float2 f = lds64(base + q);
+          set_word(v[q], 0, f.x);
+          set_word(v[q], 1, f.y);
         }
-        if (c.rg == 0) c.taus[k] = h.tau;
       }
     }
-    group_sync<GT, GPB>(c.grp);
-    // ---- trailing update: Table VI "Trailing Matrix" (Listing 7)
-    const T ct = X::conj(c.taus[k]);
+  }
+
+  // ------------------------------------------------------------ reflector
+  // xLARFG for column kn held in slot S (rows from register row I0s).
+  // Every lane of a warp that contains the owning column group computes it;
+  // only the owner's bits are used (Table VI "Column").  Branch-free, so the
+  // compiler can interleave it with the independent trailing-update FMAs.
+  template <int S, int I0s>
+  static __device__ __forceinline__ Look reflector(Ctx &c, const T (&a)[MR][NC], int kn) {
+    float s0 = 0.f, s1 = 0.f, s2 = 0.f, s3 = 0.f;
+    T alpha = X::zero();
+    const int lim = kn - c.rg;  // row r = rg + R i is below the pivot iff R i > lim
+#pragma unroll
+    for (int i = I0s; i < MR; ++i) {
+      const T x = a[i][S];
+      T xm = x;
+      if (i < I0s + Cfg::NMASK) {
+        xm = X::sel(R * i > lim, x, X::zero());
+        alpha = X::sel(R * i == lim, x, alpha);
+      }
+      switch ((i - I0s) & 3) {
+        case 0: s0 = X::abs2_acc(xm, s0); break;
+        case 1: s1 = X::abs2_acc(xm, s1); break;
+        case 2: s2 = X::abs2_acc(xm, s2); break;
+        default: s3 = X::abs2_acc(xm, s3); break;
+      }
+    }
+    float sig = (s0 + s1) + (s2 + s3);
+    sig = row_allreduce_f<R>(sig);
+    if constexpr (R > 1) alpha = X::shfl(alpha, (c.lane & ~(R - 1)) | (kn & (R - 1)));
+    const Reflector<T> h = make_reflector(alpha, sig);
+    Look l;
+    l.scal = h.scal;
+    l.tau = h.tau;
+    l.beta = h.beta;
+    return l;
+  }
+
+  // owner lanes: scale the column, store beta, publish v and tau
+  // (predicated, no divergent branch)
+  template <int S, int I0s>
+  static __device__ __forceinline__ void publish(Ctx &c, T (&a)[MR][NC], int kn, const Look &l) {
+    const bool own = c.cg == kn % G;
+    T *vb = c.vbuf + buf(kn) * VB + c.rg * MRP;
+    const int lim = kn - c.rg;
     T v[MR];
 #pragma unroll
-    for (int i = I0; i < MR; ++i) v[i] = vb[c.rg + R * i];
-    T tw[NC];
-#pragma unroll
-    for (int j = P; j < NC; ++j) {
-      T w = X::zero();
-#pragma unroll
-      for (int i = I0; i < MR; ++i) w = X::cfma(v[i], a[i][j], w);
-      w = row_allreduce<R>(w);
-      tw[j] = X::mul(ct, w);
-      if (j == P) tw[j] = X::sel(c.cg > kk, tw[j], X::zero());
+    for (int i = I0s; i < MR; ++i) {
+      const T x = a[i][S];
+      const T xs = X::mul(x, l.scal);
+      if (i < I0s + Cfg::NMASK) {
+        v[i] = X::sel(R * i > lim, xs, X::sel(R * i == lim, X::one(), X::zero()));
+        a[i][S] = X::sel(own, X::sel(R * i > lim, xs, X::sel(R * i == lim, X::make(l.beta, 0.f), x)), x);
+      } else {
+        v[i] = xs;
+        a[i][S] = X::sel(own, xs, x);
+      }
     }
 #pragma unroll
-    for (int j = P; j < NC; ++j) {
-#pragma unroll
-      for (int i = I0; i < MR; ++i) a[i][j] = X::fnms(v[i], tw[j], a[i][j]);
+    for (int q = I0s; q < MR; ++q) {
+      const int q0 = q - q % VW;
+      const bool vec_start = (q % VW == 0) && (q + VW <= MR);
+      const bool in_vec = (q % VW != 0) && (q0 >= I0s) && (q0 + VW <= MR);
+      if (vec_start) {
+        float4 f;
+        if constexpr (VW == 4) {
+          f = make_float4(X::re(v[q]), X::re(v[q + 1 < MR ? q + 1 : q]), X::re(v[q + 2 < MR ? q + 2 : q]),
+                          X::re(v[q + 3 < MR ? q + 3 : q]));
+        } else {
+          const T v1 = v[q + 1 < MR ? q + 1 : q];
+          f = make_float4(get_word(v[q], 0), get_word(v[q], 1), get_word(v1, 0), get_word(v1, 1));
+        }
+        if (own) *reinterpret_cast<float4 *>(vb + q) = f;
+      } else if (!in_vec) {
+        if (own) vb[q] = v[q];
+      }
     }
+    if (own && c.rg == 0) c.taus[kn] = l.tau;
+  }
+
+  // does this thread's warp hold the column group that owns column kn?
+  static __device__ __forceinline__ bool warp_has(const Ctx &c, int kn) {
+    if constexpr (GT <= 32) {
+      return true;
+    } else {
+      return ((kn % G) / (32 / R)) == (c.t >> 5);
+    }
+  }
+  // can this warp skip slot-P work entirely (all its column groups <= kk)?
+  static __device__ __forceinline__ bool warp_done_slot(const Ctx &c, int kk) {
+    if constexpr (GT <= 32) {
+      return false;
+    } else {
+      return ((c.t >> 5) + 1) * (32 / R) - 1 <= kk;
+    }
+  }
+
+  // ------------------------------------------------------------ trailing update
+  // Apply H_k^H (vector in vb, conj(tau) = ct) to slots [J0, J1); slot P
+  // columns with cg <= kk are excluded (already factored).  The vector is
+  // re-read from shared memory in 16-byte chunks for each pass.
+  template <int P, int I0, int J0, int J1>
+  static __device__ __forceinline__ void apply(Ctx &c, T (&a)[MR][NC], const T *vb, T ct, int kk) {
+    if constexpr (J0 < J1) {
+      constexpr int NS = J1 - J0;
+      constexpr int ACC = NS >= 4 ? 1 : (NS >= 2 ? 2 : 4);
+      T w[NS][ACC];
+#pragma unroll
+      for (int j = 0; j < NS; ++j)
+#pragma unroll
+        for (int q = 0; q < ACC; ++q) w[j][q] = X::zero();
+      {
+        T v[MR];
+        load_v<I0>(vb, v);
+#pragma unroll
+        for (int i = I0; i < MR; ++i)
+#pragma unroll
+          for (int j = 0; j < NS; ++j) w[j][(i - I0) % ACC] = X::cfma(v[i], a[i][J0 + j], w[j][(i - I0) % ACC]);
+      }
+      T tw[NS];
+#pragma unroll
+      for (int j = 0; j < NS; ++j) {
+        T s = w[j][0];
+#pragma unroll
+        for (int q = 1; q < ACC; ++q) s = X::add(s, w[j][q]);
+        s = row_allreduce<R>(s);
+        tw[j] = X::mul(ct, s);
+        if (J0 + j == P) tw[j] = X::sel(c.cg > kk, tw[j], X::zero());
+      }
+      {
+        T v[MR];
+        load_v<I0>(vb, v);
+#pragma unroll
+        for (int i = I0; i < MR; ++i)
+#pragma unroll
+          for (int j = 0; j < NS; ++j) a[i][J0 + j] = X::fnms(v[i], tw[j], a[i][J0 + j]);
+      }
+    }
+  }
+
+  // panel prologue: reflector for the panel's first column (no look-ahead
+  // across panels, which keeps one step body per panel)
+  template <int P, int I0>
+  static __device__ __forceinline__ void panel_head(Ctx &c, T (&a)[MR][NC], int k) {
+    if (warp_has(c, k)) {
+      const Look l = reflector<P, I0>(c, a, k);
+      publish<P, I0>(c, a, k, l);
+      step_arrive<GT, NBUF>(k);
+    }
+  }
+
+  // one Householder step on column k of panel P (first live register row I0):
+  // apply H_k to slot P, form + publish reflector k+1 (same slot), then apply
+  // H_k to the remaining slots while the reflector chain drains.
+  template <int P, int I0>
+  static __device__ __forceinline__ void step(Ctx &c, T (&a)[MR][NC], int k) {
+    const int kk = k - P * G;
+    if (!warp_has(c, k) || GT <= 32) step_wait<GT, NBUF>(k);
+    const T ct = X::conj(c.taus[k]);
+    const T *vb = c.vbuf + buf(k) * VB + c.rg * MRP;
+    if (!warp_done_slot(c, kk)) apply<P, I0, P, P + 1>(c, a, vb, ct, kk);
+    if (kk + 1 < G && k + 1 < c.kmax && warp_has(c, k + 1)) {
+      const Look l = reflector<P, I0>(c, a, k + 1);
+      publish<P, I0>(c, a, k + 1, l);
+      step_arrive<GT, NBUF>(k + 1);
+    }
+    apply<P, I0, P + 1, NC>(c, a, vb, ct, kk);
   }
 
   template <int P>
@@ -170,8 +366,9 @@ struct RfKernel {
       const int kbeg = P * G;
       if (kbeg >= c.kmax) return;
       const int kend = min(kbeg + G, c.kmax);
+      panel_head<P, I0>(c, a, kbeg);
 #pragma unroll 1
-      for (int k = kbeg; k < kend; ++k) column<P, I0>(c, a, k);
+      for (int k = kbeg; k < kend; ++k) step<P, I0>(c, a, k);
       panels<P + 1>(c, a);
     }
   }
@@ -180,19 +377,19 @@ struct RfKernel {
   template <int P, int I0>
   static __device__ __forceinline__ void org_column(Ctx &c, T (&a)[MR][NC], int i, const T *tau_g) {
     const int kk = i - P * G;
-    T *vb = c.vbuf + (i & 1) * MMAX;
+    T *vb = c.vbuf + buf(i) * VB + c.rg * MRP;
     const T ti = tau_g[i];
     if (c.cg == kk) {
 #pragma unroll
       for (int ii = I0; ii < MR; ++ii) {
         const int r = c.rg + R * ii;
-        vb[r] = X::sel(r > i, a[ii][P], X::sel(r == i, X::one(), X::zero()));
+        vb[ii] = X::sel(r > i, a[ii][P], X::sel(r == i, X::one(), X::zero()));
       }
     }
     group_sync<GT, GPB>(c.grp);
     T v[MR];
 #pragma unroll
-    for (int ii = I0; ii < MR; ++ii) v[ii] = vb[c.rg + R * ii];
+    for (int ii = I0; ii < MR; ++ii) v[ii] = vb[ii];
     T tw[NC];
 #pragma unroll
     for (int j = P; j < NC; ++j) {
@@ -237,6 +434,89 @@ struct RfKernel {
     }
   }
 
+  // ------------------------------------------------------------ staging
+  static __device__ __forceinline__ void load_matrix(const RfArgs &p, Ctx &c, float *smem, T *Ab, bool active,
+                                                     T (&a)[MR][NC]) {
+    const int m = p.m, n = p.n;
+    if constexpr (STAGE) {
+      float *tile = smem + Cfg::kSmallAll + c.grp * p.tileWords;
+      const float *Ag = reinterpret_cast<const float *>(Ab);
+      if (active) {
+        if (p.vec4 && p.lda == p.ldS) {
+          const int nch = (m * n) >> 2;  // contiguous matrix: linear 16-byte copy
+          for (int q = c.t; q < nch; q += GT) cp_async16(tile + 4 * q, Ag + 4 * q);
+          cp_async_wait_all();
+        } else if (p.vec4) {
+          const int mq = m >> 2;
+          for (int col = 0; col < n; ++col)
+            for (int q = c.t; q < mq; q += GT) cp_async16(tile + 4 * q + col * p.ldS, Ag + 4 * q + (long long)col * p.lda);
+          cp_async_wait_all();
+        } else {
+          for (int col = 0; col < n; ++col)
+            for (int q = c.t; q < m; q += GT) tile[q + col * p.ldS] = Ag[q + (long long)col * p.lda];
+        }
+      }
+      group_sync<GT, GPB>(c.grp);
+#pragma unroll
+      for (int i = 0; i < MR; ++i)
+#pragma unroll
+        for (int j = 0; j < NC; ++j) {
+          const int r = c.rg + R * i, col = c.cg + G * j;
+          a[i][j] = (active && r < m && col < n) ? tile[r + col * p.ldS] : 0.f;
+        }
+    } else {
+#pragma unroll
+      for (int i = 0; i < MR; ++i)
+#pragma unroll
+        for (int j = 0; j < NC; ++j) {
+          const int r = c.rg + R * i, col = c.cg + G * j;
+          a[i][j] = (active && r < m && col < n) ? Ab[r + (long long)col * p.lda] : X::zero();
+        }
+    }
+  }
+
+  static __device__ __forceinline__ void store_matrix(const RfArgs &p, Ctx &c, float *smem, T *Ab, bool active,
+                                                      const T (&a)[MR][NC]) {
+    const int m = p.m, n = p.n;
+    if constexpr (STAGE) {
+      float *tile = smem + Cfg::kSmallAll + c.grp * p.tileWords;
+      float *Ag = reinterpret_cast<float *>(Ab);
+      group_sync<GT, GPB>(c.grp);
+#pragma unroll
+      for (int i = 0; i < MR; ++i)
+#pragma unroll
+        for (int j = 0; j < NC; ++j) {
+          const int r = c.rg + R * i, col = c.cg + G * j;
+          if (r < m && col < n) tile[r + col * p.ldS] = a[i][j];
+        }
+      group_sync<GT, GPB>(c.grp);
+      if (active) {
+        if (p.vec4 && p.lda == p.ldS) {
+          const int nch = (m * n) >> 2;
+          for (int q = c.t; q < nch; q += GT)
+            *reinterpret_cast<float4 *>(Ag + 4 * q) = *reinterpret_cast<const float4 *>(tile + 4 * q);
+        } else if (p.vec4) {
+          const int mq = m >> 2;
+          for (int col = 0; col < n; ++col)
+            for (int q = c.t; q < mq; q += GT)
+              *reinterpret_cast<float4 *>(Ag + 4 * q + (long long)col * p.lda) =
+                  *reinterpret_cast<const float4 *>(tile + 4 * q + col * p.ldS);
+        } else {
+          for (int col = 0; col < n; ++col)
+            for (int q = c.t; q < m; q += GT) Ag[q + (long long)col * p.lda] = tile[q + col * p.ldS];
+        }
+      }
+    } else if (active) {
+#pragma unroll
+      for (int i = 0; i < MR; ++i)
+#pragma unroll
+        for (int j = 0; j < NC; ++j) {
+          const int r = c.rg + R * i, col = c.cg + G * j;
+          if (r < m && col < n) Ab[r + (long long)col * p.lda] = a[i][j];
+        }
+    }
+  }
+
   template <bool ORG>
   static __device__ __forceinline__ void run(const RfArgs &p) {
     extern __shared__ __align__(16) float smem[];
@@ -255,47 +535,10 @@ struct RfKernel {
     if (!active) mat = p.batch - 1;
     float *gs = smem + grp * Cfg::kSmallWords;
     c.vbuf = reinterpret_cast<T *>(gs);
-    c.taus = c.vbuf + 2 * MMAX;
+    c.taus = c.vbuf + NBUF * VB;
     T *Ab = reinterpret_cast<T *>(p.A) + mat * (long long)p.lda * p.n;
-    const int m = p.m, n = p.n;
     T a[MR][NC];
-    if constexpr (STAGE) {
-      float *tile = smem + Cfg::kSmallAll + grp * p.tileWords;
-      const float *Ag = reinterpret_cast<const float *>(Ab);
-      if (active) {
-        if (p.vec4) {
-          const int mq = m >> 2;
-          const int nch = mq * n;
-          for (int q = t; q < nch; q += GT) {
-            const int col = q / mq, rr = (q - col * mq) << 2;
-            cp_async16(tile + rr + col * p.ldS, Ag + rr + (long long)col * p.lda);
-          }
-          cp_async_wait_all();
-        } else {
-          const int nch = m * n;
-          for (int q = t; q < nch; q += GT) {
-            const int col = q / m, rr = q - col * m;
-            tile[rr + col * p.ldS] = Ag[rr + (long long)col * p.lda];
-          }
-        }
-      }
-      group_sync<GT, GPB>(grp);
-#pragma unroll
-      for (int i = 0; i < MR; ++i)
-#pragma unroll
-        for (int j = 0; j < NC; ++j) {
-          const int r = c.rg + R * i, col = c.cg + G * j;
-          a[i][j] = (active && r < m && col < n) ? tile[r + col * p.ldS] : 0.f;
-        }
-    } else {
-#pragma unroll
-      for (int i = 0; i < MR; ++i)
-#pragma unroll
-        for (int j = 0; j < NC; ++j) {
-          const int r = c.rg + R * i, col = c.cg + G * j;
-          a[i][j] = (active && r < m && col < n) ? Ab[r + (long long)col * p.lda] : X::zero();
-        }
-    }
+    load_matrix(p, c, smem, Ab, active, a);
 
     if constexpr (ORG) {
       // columns >= k start as the identity (xORG2R initialisation)
@@ -310,46 +553,11 @@ struct RfKernel {
       org_panels<NC - 1>(c, a, p.kmax, tg);
     } else {
       panels<0>(c, a);
+      group_sync<GT, GPB>(grp);  // every tau published before the tau store
     }
 
-    if constexpr (STAGE) {
-      float *tile = smem + Cfg::kSmallAll + grp * p.tileWords;
-      float *Ag = reinterpret_cast<float *>(Ab);
-#pragma unroll
-      for (int i = 0; i < MR; ++i)
-#pragma unroll
-        for (int j = 0; j < NC; ++j) {
-          const int r = c.rg + R * i, col = c.cg + G * j;
-          if (r < m && col < n) tile[r + col * p.ldS] = a[i][j];
-        }
-      group_sync<GT, GPB>(grp);
-      if (active) {
-        if (p.vec4) {
-          const int mq = m >> 2;
-          const int nch = mq * n;
-          for (int q = t; q < nch; q += GT) {
-            const int col = q / mq, rr = (q - col * mq) << 2;
-            *reinterpret_cast<float4 *>(Ag + rr + (long long)col * p.lda) =
-                *reinterpret_cast<const float4 *>(tile + rr + col * p.ldS);
-          }
-        } else {
-          const int nch = m * n;
-          for (int q = t; q < nch; q += GT) {
-            const int col = q / m, rr = q - col * m;
-            Ag[rr + (long long)col * p.lda] = tile[rr + col * p.ldS];
-          }
-        }
-      }
-    } else if (active) {
-#pragma unroll
-      for (int i = 0; i < MR; ++i)
-#pragma unroll
-        for (int j = 0; j < NC; ++j) {
-          const int r = c.rg + R * i, col = c.cg + G * j;
-          if (r < m && col < n) Ab[r + (long long)col * p.lda] = a[i][j];
-        }
-    }
-    // tau list -> global (taus complete: every column ended with a group sync)
+    store_matrix(p, c, smem, Ab, active, a);
+    // tau list -> global (each tau was published before a group barrier)
     if (!ORG && active) {
       T *tg = reinterpret_cast<T *>(p.tau) + mat * (long long)p.kmax;
       for (int idx = t; idx < p.kmax; idx += GT) tg[idx] = c.taus[idx];
@@ -358,13 +566,13 @@ struct RfKernel {
 };
 
 template <class T, int R, int G, int MR, int NC, int GPB, bool STAGE>
-__global__ void __launch_bounds__(R * G * GPB) geqrf_rf_kernel(const RfArgs p) {
+__global__ void __launch_bounds__(R * G * GPB, 1) geqrf_rf_kernel(const RfArgs p) {
   RfKernel<T, R, G, MR, NC, GPB, STAGE>::template run<false>(p);
 }
 
 // p.kmax = k (reflectors), p.n = columns of Q, p.tau read-only
 template <class T, int R, int G, int MR, int NC, int GPB, bool STAGE>
-__global__ void __launch_bounds__(R * G * GPB) orgqr_rf_kernel(const RfArgs p) {
+__global__ void __launch_bounds__(R * G * GPB, 1) orgqr_rf_kernel(const RfArgs p) {
   RfKernel<T, R, G, MR, NC, GPB, STAGE>::template run<true>(p);
 }
 
