@@ -74,9 +74,10 @@ inline int staging_ld(int m) {
   return (m + 3) & ~3;
 }
 
-template <class T, int R, int G, int MR, int NC, int GPB, bool STAGE, bool ORG>
+template <class T, int R, int G, int MR, int NC, int GPB, bool STAGE, bool EX, bool ORG>
 int launch_rf(const Call &c) {
-  using Cfg = RfCfg<T, R, G, MR, NC, GPB, STAGE>;
+  using Cfg = RfCfg<T, R, G, MR, NC, GPB, STAGE, EX>;
+  if (EX && (c.m != R * MR || c.n != G * NC)) return BQR_ERR_NOT_SUPPORTED;
   RfArgs a;
   a.A = c.A;
   a.tau = c.tau;
@@ -89,8 +90,9 @@ int launch_rf(const Call &c) {
   a.tileWords = STAGE ? ((a.ldS * c.n + 3) & ~3) : 0;
   const bool aligned = (reinterpret_cast<uintptr_t>(c.A) & 15) == 0;
   a.vec4 = (STAGE && (c.lda % 4 == 0) && (c.m % 4 == 0) && aligned) ? 1 : 0;
+  a.bulk = (STAGE && c.lda == c.m && a.ldS == c.m && aligned && ((size_t)c.m * c.n * sizeof(T)) % 16 == 0) ? 1 : 0;
   const size_t smem = (size_t)Cfg::kSmallAll * 4 + (STAGE ? (size_t)GPB * a.tileWords * 4 : 0);
-  auto kern = ORG ? orgqr_rf_kernel<T, R, G, MR, NC, GPB, STAGE> : geqrf_rf_kernel<T, R, G, MR, NC, GPB, STAGE>;
+  auto kern = ORG ? orgqr_rf_kernel<T, R, G, MR, NC, GPB, STAGE, EX> : geqrf_rf_kernel<T, R, G, MR, NC, GPB, STAGE, EX>;
   if (!ensure_smem(kern, smem)) return BQR_ERR_CUDA;
   const long long grid = (c.batch + GPB - 1) / GPB;
   if (grid > 0x7fffffffLL) return BQR_ERR_NOT_SUPPORTED;
@@ -115,11 +117,12 @@ int launch_tiny(const Call &c) {
 }
 
 // ---- size classes: smallest class that holds (m, n)
-#define RF_PLAN(T, R, G, MR, NC, GPB, STAGE, NAME)                       \
+#define RF_PLAN_X(T, R, G, MR, NC, GPB, STAGE, EX, NAME)                  \
   Plan {                                                                 \
-    NAME, &launch_rf<T, R, G, MR, NC, GPB, STAGE, false>,                \
-        &launch_rf<T, R, G, MR, NC, GPB, STAGE, true>                    \
+    NAME, &launch_rf<T, R, G, MR, NC, GPB, STAGE, EX, false>,            \
+        &launch_rf<T, R, G, MR, NC, GPB, STAGE, EX, true>                \
   }
+#define RF_PLAN(T, R, G, MR, NC, GPB, STAGE, NAME) RF_PLAN_X(T, R, G, MR, NC, GPB, STAGE, false, NAME)
 
 struct ClassEntry {
   bqr_dtype_t dt;
@@ -133,13 +136,14 @@ struct ClassEntry {
 // then the smallest class that holds (m, n).
 const ClassEntry kClasses[] = {
     // headline shapes, exact fits
-    {BQR_R32, 56, 56, 56, 56, false, RF_PLAN(float, 2, 8, 28, 7, 2, true, "rf_f32_R2G8_28x7_x2_stage")},
-    {BQR_C64, 240, 66, 240, 66, false, RF_PLAN(float2, 16, 22, 15, 3, 1, false, "rf_c64_R16G22_15x3_cta")},
+    {BQR_R32, 56, 56, 56, 56, false, RF_PLAN_X(float, 2, 8, 28, 7, 2, true, true, "rf_f32_R2G8_28x7_x2_exact")},
+    {BQR_R32, 56, 56, 56, 56, true, RF_PLAN(float, 2, 8, 28, 7, 2, true, "rf_f32_R2G8_28x7_x2_stage")},
+    {BQR_C64, 240, 66, 240, 66, false, RF_PLAN(float2, 32, 11, 8, 6, 1, false, "rf_c64_R32G11_8x6_cta")},
+    {BQR_C64, 240, 66, 240, 66, true, RF_PLAN(float2, 16, 22, 15, 3, 1, false, "rf_c64_R16G22_15x3_cta")},
     // alternatives kept for measurement (BQR_FORCE_VARIANT)
     {BQR_R32, 56, 56, 56, 56, true, RF_PLAN(float, 4, 8, 14, 7, 1, true, "rf_f32_R4G8_14x7_x1_stage")},
     {BQR_R32, 56, 56, 56, 56, true, RF_PLAN(float, 4, 4, 14, 14, 2, true, "rf_f32_R4G4_14x14_x2_stage")},
     {BQR_C64, 240, 66, 240, 66, true, RF_PLAN(float2, 32, 16, 8, 5, 1, false, "rf_c64_R32G16_8x5_cta")},
-    {BQR_C64, 256, 66, 240, 66, true, RF_PLAN(float2, 32, 11, 8, 6, 1, false, "rf_c64_R32G11_8x6_cta")},
     // fp32 classes
     {BQR_R32, 16, 16, 0, 0, false, RF_PLAN(float, 2, 4, 8, 4, 8, true, "rf_f32_R2G4_8x4_x8_stage")},
     {BQR_R32, 32, 32, 0, 0, false, RF_PLAN(float, 2, 8, 16, 4, 4, true, "rf_f32_R2G8_16x4_x4_stage")},

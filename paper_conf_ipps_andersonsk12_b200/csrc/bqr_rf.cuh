@@ -43,12 +43,19 @@ struct RfArgs {
   int ldS;        // staging tile leading dimension (elements)
   int tileWords;  // staging tile stride per group (32-bit words)
   int vec4;       // 16-byte vectorised staging legal (lda%4==0, m%4==0, aligned)
+  int bulk;       // contiguous matrices (lda == m), 16-byte aligned, size % 16 == 0:
+                  // stage with one TMA bulk copy per matrix each way
 };
+
+// Warp barrier as opaque PTX: nvcc versions the whole rest of a kernel on
+// "was the warp diverged at this __syncwarp()" (BRA.DIV + a full copy of the
+// factorisation); the asm form keeps one copy.
+__device__ __forceinline__ void warp_sync() { asm volatile("bar.warp.sync -1;" ::: "memory"); }
 
 template <int GT, int GPB>
 __device__ __forceinline__ void group_sync(int grp) {
   if constexpr (GT <= 32) {
-    __syncwarp();
+    warp_sync();
   } else if constexpr (GPB == 1) {
     __syncthreads();
   } else {
@@ -64,13 +71,13 @@ __device__ __forceinline__ void group_sync(int grp) {
 // buffers) keep an early arrival off an instance that has not completed.
 template <int GT, int NB>
 __device__ __forceinline__ void step_arrive(int k) {
-  __syncwarp();
+  warp_sync();
   if constexpr (GT > 32) asm volatile("bar.arrive %0, %1;" ::"r"(1 + k % NB), "r"(GT) : "memory");
 }
 template <int GT, int NB>
 __device__ __forceinline__ void step_wait(int k) {
   if constexpr (GT <= 32) {
-    __syncwarp();
+    warp_sync();
   } else {
     asm volatile("bar.sync %0, %1;" ::"r"(1 + k % NB), "r"(GT) : "memory");
   }
@@ -81,6 +88,42 @@ __device__ __forceinline__ void cp_async16(void *smem_dst, const void *gmem_src)
   asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(s), "l"(gmem_src) : "memory");
 }
 __device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;\n" ::: "memory"); }
+
+// TMA bulk copies (cp.async.bulk) completing on an mbarrier / bulk group.
+__device__ __forceinline__ unsigned smem_u32(const void *p) { return (unsigned)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init(void *bar, unsigned count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void bulk_load(void *dst, const void *src, unsigned bytes, void *bar) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                   smem_u32(dst)),
+               "l"(src), "r"(bytes), "r"(smem_u32(bar))
+               : "memory");
+}
+// One bounded hardware wait (suspend-time hint); the retry loop is plain
+// C++ so the compiler sees structured control flow (an asm-internal branch
+// makes it assume the warp may stay diverged and duplicate the whole kernel
+// behind a BRA.DIV).
+__device__ __forceinline__ bool mbar_try_wait(void *bar, unsigned parity) {
+  unsigned ok;
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2, %3;\n\t"
+      "selp.u32 %0, 1, 0, p;\n}"
+      : "=r"(ok)
+      : "r"(smem_u32(bar)), "r"(parity), "r"(1000000u)
+      : "memory");
+  return ok != 0;
+}
+__device__ __forceinline__ void bulk_store(void *dst, const void *src, unsigned bytes) {
+  asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(dst), "r"(smem_u32(src)), "r"(bytes)
+               : "memory");
+  asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+}
+__device__ __forceinline__ void bulk_store_drain() { asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); }
+__device__ __forceinline__ void fence_async_smem() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
 
 // 16-byte shared loads that the compiler may not merge across passes (keeps
 // the Householder vector out of the register file between the
@@ -104,7 +147,7 @@ __device__ __forceinline__ float2 lds64(const void *p) {
   return v;
 }
 
-template <class T, int R, int G, int MR, int NC, int GPB, bool STAGE>
+template <class T, int R, int G, int MR, int NC, int GPB, bool STAGE, bool EX = false>
 struct RfCfg {
   static constexpr int GT = R * G;
   static constexpr int NT = GT * GPB;
@@ -125,30 +168,38 @@ struct RfCfg {
   // multi-warp groups publish ahead without a full barrier (see step_arrive)
   static constexpr int NBUF = GT <= 32 ? 2 : 32 / R + 2;
   static_assert(GT <= 32 || GPB == 1, "multi-warp groups: one group per CTA");
-  static constexpr int kSmallWords = ((NBUF * VB + NMAX) * E + 3) / 4 * 4;
+  // [NBUF][VB] vectors | [NMAX] taus | mbarrier (8-byte aligned, 4 words)
+  static constexpr int kMbarWord = ((NBUF * VB + NMAX) * E + 3) / 4 * 4;
+  static constexpr int kSmallWords = kMbarWord + 4;
   static constexpr int kSmallAll = ((GPB * kSmallWords + 31) / 32) * 32;
   static_assert(R >= 1 && R <= 32 && (R & (R - 1)) == 0, "R must be a power of two <= 32");
   static_assert(GT <= 32 ? (32 % GT == 0) : (GT % 32 == 0 && 32 % R == 0), "group must tile warps");
   static_assert(!STAGE || E == 1, "smem staging implemented for fp32");
   // register rows that may hold the pivot row of a column inside one panel
-  static constexpr int NMASK = (G + R - 1) / R + 1;
+  static constexpr int NMASK = (G % R == 0) ? G / R : (G + R - 1) / R + 1;
 };
 
-template <class T, int R, int G, int MR, int NC, int GPB, bool STAGE>
+template <class T, int R, int G, int MR, int NC, int GPB, bool STAGE, bool EX = false>
 struct RfKernel {
-  using Cfg = RfCfg<T, R, G, MR, NC, GPB, STAGE>;
+  using Cfg = RfCfg<T, R, G, MR, NC, GPB, STAGE, EX>;
   using X = El<T>;
   static constexpr int GT = Cfg::GT;
   static constexpr int VW = Cfg::VW;
   static constexpr int MRP = Cfg::MRP;
   static constexpr int VB = Cfg::VB;
   static constexpr int NBUF = Cfg::NBUF;
+  static constexpr int MMAX_ = Cfg::MMAX, NMAX_ = Cfg::NMAX;
+  // Fully unrolled column loop: ~27% fewer instructions for 56x56, but the
+  // ~250 KB of straight-line code thrashes the instruction cache (58% of
+  // stall samples "no_inst" on B200), so the panel loop is the default.
+  static constexpr bool kFullUnroll = false;
   static __device__ __forceinline__ int buf(int k) { return k % NBUF; }
 
   struct Ctx {
     T *vbuf;   // [NBUF][VB]
     T *taus;   // [NMAX]
     int rg, cg, t, lane, grp;
+    int wid;   // warp index in the group, warp-uniform by construction (shfl)
     int kmax;
   };
 
@@ -228,24 +279,28 @@ struct RfKernel {
     return l;
   }
 
-  // owner lanes: scale the column, store beta, publish v and tau
-  // (predicated, no divergent branch)
+  // Owner lanes (own && on): scale the column, store beta, publish v and
+  // tau.  Branch-free, so no divergent region precedes the next shuffles
+  // (a divergent branch makes the compiler guard every later shuffle with
+  // WARPSYNC): non-owner lanes multiply by 1 (bit-exact no-op) and only the
+  // few rows that can hold the pivot need selects.
   template <int S, int I0s>
-  static __device__ __forceinline__ void publish(Ctx &c, T (&a)[MR][NC], int kn, const Look &l) {
-    const bool own = c.cg == kn % G;
+  static __device__ __forceinline__ void publish(Ctx &c, T (&a)[MR][NC], int kn, const Look &l, bool on) {
+    const bool own = on && ((GT > 32 && R == 32) ? true : (c.cg == kn % G));
+    const T scal = X::sel(own, l.scal, X::one());
     T *vb = c.vbuf + buf(kn) * VB + c.rg * MRP;
     const int lim = kn - c.rg;
     T v[MR];
 #pragma unroll
     for (int i = I0s; i < MR; ++i) {
       const T x = a[i][S];
-      const T xs = X::mul(x, l.scal);
+      const T xs = X::mul(x, scal);
       if (i < I0s + Cfg::NMASK) {
         v[i] = X::sel(R * i > lim, xs, X::sel(R * i == lim, X::one(), X::zero()));
-        a[i][S] = X::sel(own, X::sel(R * i > lim, xs, X::sel(R * i == lim, X::make(l.beta, 0.f), x)), x);
+        a[i][S] = X::sel(R * i > lim, xs, X::sel(own && R * i == lim, X::make(l.beta, 0.f), x));
       } else {
         v[i] = xs;
-        a[i][S] = X::sel(own, xs, x);
+        a[i][S] = xs;
       }
     }
 #pragma unroll
@@ -275,7 +330,7 @@ struct RfKernel {
     if constexpr (GT <= 32) {
       return true;
     } else {
-      return ((kn % G) / (32 / R)) == (c.t >> 5);
+      return ((kn % G) / (32 / R)) == c.wid;
     }
   }
   // can this warp skip slot-P work entirely (all its column groups <= kk)?
@@ -283,7 +338,7 @@ struct RfKernel {
     if constexpr (GT <= 32) {
       return false;
     } else {
-      return ((c.t >> 5) + 1) * (32 / R) - 1 <= kk;
+      return (c.wid + 1) * (32 / R) - 1 <= kk;
     }
   }
 
@@ -295,7 +350,9 @@ struct RfKernel {
   static __device__ __forceinline__ void apply(Ctx &c, T (&a)[MR][NC], const T *vb, T ct, int kk) {
     if constexpr (J0 < J1) {
       constexpr int NS = J1 - J0;
-      constexpr int ACC = NS >= 4 ? 1 : (NS >= 2 ? 2 : 4);
+      // 4 partial sums per slot: ptxas walks the slots one after another, so
+      // a single accumulator per slot is a 4-cycle-per-row serial chain
+      constexpr int ACC = 4;
       T w[NS][ACC];
 #pragma unroll
       for (int j = 0; j < NS; ++j)
@@ -336,7 +393,7 @@ struct RfKernel {
   static __device__ __forceinline__ void panel_head(Ctx &c, T (&a)[MR][NC], int k) {
     if (warp_has(c, k)) {
       const Look l = reflector<P, I0>(c, a, k);
-      publish<P, I0>(c, a, k, l);
+      publish<P, I0>(c, a, k, l, true);
       step_arrive<GT, NBUF>(k);
     }
   }
@@ -351,12 +408,169 @@ struct RfKernel {
     const T ct = X::conj(c.taus[k]);
     const T *vb = c.vbuf + buf(k) * VB + c.rg * MRP;
     if (!warp_done_slot(c, kk)) apply<P, I0, P, P + 1>(c, a, vb, ct, kk);
-    if (kk + 1 < G && k + 1 < c.kmax && warp_has(c, k + 1)) {
+    const bool la = kk + 1 < G && k + 1 < c.kmax && warp_has(c, k + 1);
+    if constexpr (GT <= 32) {
+      // sub-warp groups: the reflector chain (computed unconditionally, no
+      // branch around its shuffles) overlaps the remaining updates in one
+      // basic block; the owner lanes publish at the end of the step
       const Look l = reflector<P, I0>(c, a, k + 1);
-      publish<P, I0>(c, a, k + 1, l);
-      step_arrive<GT, NBUF>(k + 1);
+      apply<P, I0, P + 1, NC>(c, a, vb, ct, kk);
+      publish<P, I0>(c, a, k + 1, l, la);
+    } else {
+      // multi-warp groups: publish first so the other warps never wait
+      if (la) {
+        const Look l = reflector<P, I0>(c, a, k + 1);
+        publish<P, I0>(c, a, k + 1, l, true);
+        step_arrive<GT, NBUF>(k + 1);
+      }
+      apply<P, I0, P + 1, NC>(c, a, vb, ct, kk);
     }
-    apply<P, I0, P + 1, NC>(c, a, vb, ct, kk);
+  }
+
+  // ====================================================================
+  // Fully unrolled variant (UNR): the column index is a compile-time
+  // constant after unrolling, so row ranges are exact (no panel waste) and
+  // almost every pivot mask folds away; only the lane-dependent row offset
+  // rg and the slot-mask cg > kk remain runtime.  Used for sub-warp groups of
+  // exact-shape classes (e.g. 2 x 56x56 fp32 per warp), where the masks and
+  // panel waste were ~30% of all issued instructions.
+  // ====================================================================
+  // r = rg + R i vs the pivot kn (folds to a constant unless i straddles kn)
+  static __device__ __forceinline__ bool row_gt(const Ctx &c, int i, int kn) {
+    return (R * i > kn) ? true : ((R * i + R - 1 <= kn) ? false : (R * i > kn - c.rg));
+  }
+  static __device__ __forceinline__ bool row_eq(const Ctx &c, int i, int kn) {
+    return (R * i > kn || R * i + R - 1 < kn) ? false : (R * i == kn - c.rg);
+  }
+
+  static __device__ __forceinline__ Look ureflector(Ctx &c, const T (&a)[MR][NC], int kn, int S) {
+    float s0 = 0.f, s1 = 0.f, s2 = 0.f, s3 = 0.f;
+    T alpha = X::zero();
+    const int i0 = kn / R;
+#pragma unroll
+    for (int i = 0; i < MR; ++i) {
+      if (i < i0) continue;
+      const T x = a[i][S];
+      const T xm = X::sel(row_gt(c, i, kn), x, X::zero());
+      alpha = X::sel(row_eq(c, i, kn), x, alpha);
+      switch ((i - i0) & 3) {
+        case 0: s0 = X::abs2_acc(xm, s0); break;
+        case 1: s1 = X::abs2_acc(xm, s1); break;
+        case 2: s2 = X::abs2_acc(xm, s2); break;
+        default: s3 = X::abs2_acc(xm, s3); break;
+      }
+    }
+    float sig = (s0 + s1) + (s2 + s3);
+    sig = row_allreduce_f<R>(sig);
+    if constexpr (R > 1) alpha = X::shfl(alpha, (c.lane & ~(R - 1)) | (kn & (R - 1)));
+    const Reflector<T> h = make_reflector(alpha, sig);
+    Look l;
+    l.scal = h.scal;
+    l.tau = h.tau;
+    l.beta = h.beta;
+    return l;
+  }
+
+  static __device__ __forceinline__ void upublish(Ctx &c, T (&a)[MR][NC], int kn, int S, const Look &l) {
+    const bool own = c.cg == kn % G;
+    const T scal = X::sel(own, l.scal, X::one());
+    T *vb = c.vbuf + buf(kn) * VB + c.rg * MRP;
+    const int i0 = kn / R;
+#pragma unroll
+    for (int i = 0; i < MR; ++i) {
+      if (i < i0) continue;
+      const T x = a[i][S];
+      const T xs = X::mul(x, scal);
+      const bool gt = row_gt(c, i, kn), eq = row_eq(c, i, kn);
+      const T v = X::sel(gt, xs, X::sel(eq, X::one(), X::zero()));
+      a[i][S] = X::sel(gt, xs, X::sel(own && eq, X::make(l.beta, 0.f), x));
+      if (own) vb[i] = v;
+    }
+    if (own && c.rg == 0) c.taus[kn] = l.tau;
+  }
+
+  // H_k^H applied to slots [J0, J1) over register rows [i0, MR)
+  static __device__ __forceinline__ void uapply(Ctx &c, T (&a)[MR][NC], const T *vb, T ct, int k, int J0, int J1) {
+    const int P = k / G, kk = k % G, i0 = k / R;
+    const int NS = J1 - J0;
+    if (NS <= 0) return;
+    const int ACC = NS >= 4 ? 1 : (NS >= 2 ? 2 : 4);
+    T w[NC][4];
+#pragma unroll
+    for (int j = 0; j < NC; ++j)
+#pragma unroll
+      for (int q = 0; q < 4; ++q) w[j][q] = X::zero();
+#pragma unroll
+    for (int i = 0; i < MR; ++i) {
+      if (i < i0) continue;
+      const T v = vb[i];
+#pragma unroll
+      for (int j = 0; j < NC; ++j) {
+        if (j < J0 || j >= J1) continue;
+        w[j][(i - i0) % ACC] = X::cfma(v, a[i][j], w[j][(i - i0) % ACC]);
+      }
+    }
+    T tw[NC];
+#pragma unroll
+    for (int j = 0; j < NC; ++j) {
+      if (j < J0 || j >= J1) continue;
+      T s = w[j][0];
+#pragma unroll
+      for (int q = 1; q < 4; ++q)
+        if (q < ACC) s = X::add(s, w[j][q]);
+      s = row_allreduce<R>(s);
+      tw[j] = X::mul(ct, s);
+      if (j == P) tw[j] = X::sel(c.cg > kk, tw[j], X::zero());
+    }
+    asm volatile("" ::: "memory");  // re-read v for the update (keeps it out of registers)
+#pragma unroll
+    for (int i = 0; i < MR; ++i) {
+      if (i < i0) continue;
+      const T v = vb[i];
+#pragma unroll
+      for (int j = 0; j < NC; ++j) {
+        if (j < J0 || j >= J1) continue;
+        a[i][j] = X::fnms(v, tw[j], a[i][j]);
+      }
+    }
+  }
+
+  template <int K>
+  static __device__ __forceinline__ void ustep(Ctx &c, T (&a)[MR][NC], int kmax) {
+    constexpr int P = K / G, kk = K % G;
+    constexpr int lo = (kk == G - 1) ? P + 1 : P;
+    step_wait<GT, NBUF>(K);
+    const T ct = X::conj(c.taus[K]);
+    const T *vb = c.vbuf + buf(K) * VB + c.rg * MRP;
+    // live slots [lo, NC); slot lo holds column K+1: H_K on it first, then
+    // reflector K+1 (unconditional: no branch around its shuffles), then the
+    // remaining slots while the reflector chain drains, then the owner lanes
+    // publish v_{K+1}
+    if constexpr (lo < NC) {
+      uapply(c, a, vb, ct, K, lo, lo + 1);
+      const Look l = ureflector(c, a, K + 1, lo);
+      uapply(c, a, vb, ct, K, lo + 1, NC);
+      if (K + 1 < kmax) upublish(c, a, K + 1, lo, l);
+    }
+  }
+
+  template <int K>
+  static __device__ __forceinline__ void usteps(Ctx &c, T (&a)[MR][NC], int kmax) {
+    if constexpr (K < NMAX_ && K < MMAX_) {
+      if (EX || K < kmax) {
+        ustep<K>(c, a, kmax);
+        usteps<K + 1>(c, a, kmax);
+      }
+    }
+  }
+
+  static __device__ __forceinline__ void ufactor(Ctx &c, T (&a)[MR][NC]) {
+    const int kmax = EX ? (MMAX_ < NMAX_ ? MMAX_ : NMAX_) : c.kmax;
+    {
+      const Look l = ureflector(c, a, 0, 0);
+      if (kmax > 0) upublish(c, a, 0, 0, l);
+    }
+    usteps<0>(c, a, kmax);
   }
 
   template <int P>
@@ -435,13 +649,40 @@ struct RfKernel {
   }
 
   // ------------------------------------------------------------ staging
+  // in-bounds test; compile-time true for exact-shape instantiations
+  static __device__ __forceinline__ bool inb(int r, int col, int m, int n) {
+    if constexpr (EX) return true;
+    return r < m && col < n;
+  }
+
   static __device__ __forceinline__ void load_matrix(const RfArgs &p, Ctx &c, float *smem, T *Ab, bool active,
                                                      T (&a)[MR][NC]) {
     const int m = p.m, n = p.n;
     if constexpr (STAGE) {
       float *tile = smem + Cfg::kSmallAll + c.grp * p.tileWords;
       const float *Ag = reinterpret_cast<const float *>(Ab);
-      if (active) {
+      if (p.bulk) {
+        // one TMA bulk copy of the whole (contiguous) matrix
+        void *bar = smem + c.grp * Cfg::kSmallWords + Cfg::kMbarWord;
+        if (c.t == 0) mbar_init(bar, 1);
+        group_sync<GT, GPB>(c.grp);
+        if (c.t == 0 && active) bulk_load(tile, Ag, (unsigned)(m * n * 4), bar);
+        // every lane waits on the barriers of ALL groups sharing its warp, so
+        // the warp leaves the loop converged (per-group exits would leave the
+        // two matrices of a warp running diverged for the whole kernel)
+        constexpr int GPW = GT <= 32 ? 32 / GT : 1;
+        const int g0 = GT <= 32 ? (c.grp / GPW) * GPW : c.grp;
+        bool done = false;
+        while (!done) {
+          done = true;
+#pragma unroll
+          for (int g = 0; g < GPW; ++g) {
+            void *bg = smem + (g0 + g) * Cfg::kSmallWords + Cfg::kMbarWord;
+            const long long mg = (long long)blockIdx.x * GPB + g0 + g;
+            if (mg < p.batch) done = mbar_try_wait(bg, 0) && done;
+          }
+        }
+      } else if (active) {
         if (p.vec4 && p.lda == p.ldS) {
           const int nch = (m * n) >> 2;  // contiguous matrix: linear 16-byte copy
           for (int q = c.t; q < nch; q += GT) cp_async16(tile + 4 * q, Ag + 4 * q);
@@ -457,12 +698,13 @@ struct RfKernel {
         }
       }
       group_sync<GT, GPB>(c.grp);
+      const int ld = EX ? R * MR : p.ldS;
 #pragma unroll
       for (int i = 0; i < MR; ++i)
 #pragma unroll
         for (int j = 0; j < NC; ++j) {
           const int r = c.rg + R * i, col = c.cg + G * j;
-          a[i][j] = (active && r < m && col < n) ? tile[r + col * p.ldS] : 0.f;
+          a[i][j] = (inb(r, col, m, n) && (EX || active)) ? tile[r + col * ld] : 0.f;
         }
     } else {
 #pragma unroll
@@ -470,7 +712,7 @@ struct RfKernel {
 #pragma unroll
         for (int j = 0; j < NC; ++j) {
           const int r = c.rg + R * i, col = c.cg + G * j;
-          a[i][j] = (active && r < m && col < n) ? Ab[r + (long long)col * p.lda] : X::zero();
+          a[i][j] = (active && inb(r, col, m, n)) ? Ab[r + (long long)col * p.lda] : X::zero();
         }
     }
   }
@@ -481,14 +723,28 @@ struct RfKernel {
     if constexpr (STAGE) {
       float *tile = smem + Cfg::kSmallAll + c.grp * p.tileWords;
       float *Ag = reinterpret_cast<float *>(Ab);
+      const int ld = EX ? R * MR : p.ldS;
       group_sync<GT, GPB>(c.grp);
 #pragma unroll
       for (int i = 0; i < MR; ++i)
 #pragma unroll
         for (int j = 0; j < NC; ++j) {
           const int r = c.rg + R * i, col = c.cg + G * j;
-          if (r < m && col < n) tile[r + col * p.ldS] = a[i][j];
+          if (inb(r, col, m, n)) tile[r + col * ld] = a[i][j];
         }
+      // opaque copy of the flag: keeps the compiler from duplicating the whole
+      // factorisation to thread the load-time branch into the store
+      int bulk;
+      asm volatile("mov.b32 %0, %1;" : "=r"(bulk) : "r"(p.bulk));
+      if (bulk) {
+        fence_async_smem();
+        group_sync<GT, GPB>(c.grp);
+        if (c.t == 0 && active) {
+          bulk_store(Ag, tile, (unsigned)(m * n * 4));
+          bulk_store_drain();
+        }
+        return;
+      }
       group_sync<GT, GPB>(c.grp);
       if (active) {
         if (p.vec4 && p.lda == p.ldS) {
@@ -512,7 +768,7 @@ struct RfKernel {
 #pragma unroll
         for (int j = 0; j < NC; ++j) {
           const int r = c.rg + R * i, col = c.cg + G * j;
-          if (r < m && col < n) Ab[r + (long long)col * p.lda] = a[i][j];
+          if (inb(r, col, m, n)) Ab[r + (long long)col * p.lda] = a[i][j];
         }
     }
   }
@@ -529,6 +785,7 @@ struct RfKernel {
     c.rg = t % R;
     c.cg = t / R;
     c.lane = tid & 31;
+    c.wid = __shfl_sync(0xffffffffu, t >> 5, 0);
     c.kmax = p.kmax;
     long long mat = (long long)blockIdx.x * GPB + grp;
     const bool active = mat < p.batch;
@@ -552,7 +809,11 @@ struct RfKernel {
       const T *tg = reinterpret_cast<const T *>(p.tau) + mat * (long long)p.kmax;
       org_panels<NC - 1>(c, a, p.kmax, tg);
     } else {
-      panels<0>(c, a);
+      if constexpr (kFullUnroll && EX && GT <= 32) {
+        ufactor(c, a);
+      } else {
+        panels<0>(c, a);
+      }
       group_sync<GT, GPB>(grp);  // every tau published before the tau store
     }
 
@@ -565,15 +826,15 @@ struct RfKernel {
   }
 };
 
-template <class T, int R, int G, int MR, int NC, int GPB, bool STAGE>
+template <class T, int R, int G, int MR, int NC, int GPB, bool STAGE, bool EX>
 __global__ void __launch_bounds__(R * G * GPB, 1) geqrf_rf_kernel(const RfArgs p) {
-  RfKernel<T, R, G, MR, NC, GPB, STAGE>::template run<false>(p);
+  RfKernel<T, R, G, MR, NC, GPB, STAGE, EX>::template run<false>(p);
 }
 
 // p.kmax = k (reflectors), p.n = columns of Q, p.tau read-only
-template <class T, int R, int G, int MR, int NC, int GPB, bool STAGE>
+template <class T, int R, int G, int MR, int NC, int GPB, bool STAGE, bool EX>
 __global__ void __launch_bounds__(R * G * GPB, 1) orgqr_rf_kernel(const RfArgs p) {
-  RfKernel<T, R, G, MR, NC, GPB, STAGE>::template run<true>(p);
+  RfKernel<T, R, G, MR, NC, GPB, STAGE, EX>::template run<true>(p);
 }
 
 }  // namespace bqr
