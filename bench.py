@@ -34,6 +34,7 @@ sys.path.insert(0, ROOT)
 
 import numpy as np  # noqa: E402
 
+import bqr_dist  # noqa: E402
 import bqr_inputs  # noqa: E402
 import bqr_metrics as bm  # noqa: E402
 
@@ -44,8 +45,7 @@ PROFILE_TRAFFIC = os.path.join(ROOT, "profiles", "traffic.json")
 
 # --------------------------------------------------------------------- utils
 
-def env_rank():
-    return int(os.environ.get("RANK", 0)), int(os.environ.get("WORLD_SIZE", 1)), int(os.environ.get("LOCAL_RANK", 0))
+env_rank = bqr_dist.env_rank
 
 
 class ClockSampler:
@@ -128,7 +128,7 @@ class Workload:
         self.nrhs = cfg.get("nrhs", 0)
         self.torch, self.bqr = torch, bqr
         # weak scaling: rank r owns matrices [r*B, (r+1)*B) of a world*B seeded stream
-        lo, hi = rank * self.batch, (rank + 1) * self.batch
+        lo, hi = bqr_dist.rank_slice(rank, world, self.batch)
         host = bqr_inputs.random_batch(self.m, self.n, world * self.batch, self.dt, cfg["seed"], cfg["dist"],
                                        start=lo, stop=hi)
         self.host = host
@@ -177,18 +177,11 @@ class Workload:
 
 
 def barrier(torch, dist, world):
-    torch.cuda.synchronize()
-    if world > 1:
-        dist.barrier()
-    torch.cuda.synchronize()
+    bqr_dist.barrier(torch, dist)
 
 
 def max_over_ranks(torch, dist, world, x: float) -> float:
-    if world == 1:
-        return x
-    t = torch.tensor([x], dtype=torch.float64, device="cuda")
-    dist.all_reduce(t, op=dist.ReduceOp.MAX)
-    return float(t.item())
+    return bqr_dist.max_over_ranks(torch, dist, x)
 
 
 def time_workload(w: Workload, steps: int, warmup: int, torch, dist, world, flush, sampler=None):
@@ -359,6 +352,13 @@ def run_ours(args):
             out["gpu_launches"] += k2 * (2 if w.nrhs else 1)
             del w
         out["also"] = also
+    # determinism evidence (outside the timed region): checksum of one
+    # factorised slice per rank, gathered over the process group
+    main.restore()
+    main.geqrf()
+    torch.cuda.synchronize()
+    sums = bqr_dist.gather_ints(torch, dist, [bqr_dist.checksum(main.A.cpu().numpy())])
+    out["checksums"] = [s[0] for s in sums]
     if rank == 0 and world == 1 and not args.no_cpu:
         out["cpu_baseline"] = cpu_baseline(args.config)
     if rank == 0:

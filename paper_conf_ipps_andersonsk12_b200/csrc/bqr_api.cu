@@ -225,12 +225,13 @@ bool orgqr_plan(bqr_dtype_t dt, int m, int n, Plan *out) {
 
 template <class T, int MR, int NB>
 int launch_apply(const ApplyArgs &a, cudaStream_t s) {
-  using K = ApplyQh<T, MR, NB>;
+  constexpr int PF = MR <= 2 ? 8 : 6;  // reflector columns in flight per warp
+  using K = ApplyQh<T, MR, NB, PF>;
   const long long nblk = (a.nrhs + NB - 1) / NB;
   const long long items = a.batch * nblk;
   const long long grid = (items + K::kWarps - 1) / K::kWarps;
   if (grid > 0x7fffffffLL) return BQR_ERR_NOT_SUPPORTED;
-  apply_qh_kernel<T, MR, NB><<<(unsigned)grid, K::kWarps * 32, 0, s>>>(a);
+  apply_qh_kernel<T, MR, NB, PF><<<(unsigned)grid, K::kWarps * 32, 0, s>>>(a);
   return finish_launch();
 }
 

@@ -6,9 +6,11 @@
 //
 // One warp per (matrix, block of NB right-hand sides): rows are cyclic over
 // the 32 lanes (each warp access to a reflector column is a contiguous,
-// coalesced segment), the NB dot products v^H B are warp-shuffle butterflies
-// (no barrier), and the next reflector column is prefetched into registers
-// while the current one is applied (V does not depend on B).
+// coalesced segment) and the NB dot products v^H B are warp-shuffle
+// butterflies (no barrier).  V does not depend on B, so the reflector
+// columns stream through a PF-deep register ring: column i+PF is requested
+// while column i is applied, which hides the L2/HBM latency behind the
+// serial chain of reflector applications.
 #pragma once
 #include "bqr_common.cuh"
 
@@ -22,18 +24,40 @@ struct ApplyArgs {
   int lda, ncolsA, m, k, nrhs, ldb;
 };
 
-template <class T, int MR, int NB>
+template <class T, int MR, int NB, int PF>
 struct ApplyQh {
   using X = El<T>;
-  static constexpr int kWarps = 4;
+  static constexpr int kWarps = MR >= 4 ? 1 : 4;  // long columns: one warp per CTA spreads the SMs
 
+  // raw column (rows >= i); the v_i = 1 / zero-above masks are applied at
+  // use time, so nothing consumes the load until the ring comes round
   static __device__ __forceinline__ void load_v(T (&v)[MR], const T *col, int i, int m, int lane) {
 #pragma unroll
     for (int s = 0; s < MR; ++s) {
       const int r = lane + 32 * s;
-      T x = X::zero();
-      if (r > i && r < m) x = col[r];
-      v[s] = X::sel(r == i, X::one(), x);
+      if (r >= i && r < m) v[s] = col[r];
+    }
+  }
+
+  static __device__ __forceinline__ void apply_one(T (&b)[MR][NB], const T (&raw)[MR], T ct, int i, int m, int lane) {
+    T v[MR];
+#pragma unroll
+    for (int s = 0; s < MR; ++s) {
+      const int r = lane + 32 * s;
+      v[s] = X::sel(r > i && r < m, raw[s], X::sel(r == i, X::one(), X::zero()));
+    }
+#pragma unroll
+    for (int j = 0; j < NB; ++j) {
+      T w0 = X::zero(), w1 = X::zero();
+#pragma unroll
+      for (int s = 0; s < MR; ++s) {
+        if (s & 1) w1 = X::cfma(v[s], b[s][j], w1);
+        else w0 = X::cfma(v[s], b[s][j], w0);
+      }
+      const T w = row_allreduce<32>(X::add(w0, w1));
+      const T tw = X::mul(ct, w);
+#pragma unroll
+      for (int s = 0; s < MR; ++s) b[s][j] = X::fnms(v[s], tw, b[s][j]);
     }
   }
 
@@ -55,24 +79,34 @@ struct ApplyQh {
         const int r = lane + 32 * s;
         b[s][j] = (r < p.m && j0 + j < p.nrhs) ? Bb[r + (long long)(j0 + j) * p.ldb] : X::zero();
       }
-    T v[MR], vn[MR];
-    if (p.k > 0) load_v(v, Ab, 0, p.m, lane);
-#pragma unroll 1
-    for (int i = 0; i < p.k; ++i) {
-      if (i + 1 < p.k) load_v(vn, Ab + (long long)(i + 1) * p.lda, i + 1, p.m, lane);
-      const T ct = X::conj(tg[i]);
+    T ring[PF][MR];
+    T tr[PF];
 #pragma unroll
-      for (int j = 0; j < NB; ++j) {
-        T w = X::zero();
+    for (int q = 0; q < PF; ++q) {
 #pragma unroll
-        for (int s = 0; s < MR; ++s) w = X::cfma(v[s], b[s][j], w);
-        w = row_allreduce<32>(w);
-        const T tw = X::mul(ct, w);
+      for (int s = 0; s < MR; ++s) ring[q][s] = X::zero();
+      tr[q] = X::zero();
+    }
 #pragma unroll
-        for (int s = 0; s < MR; ++s) b[s][j] = X::fnms(v[s], tw, b[s][j]);
+    for (int q = 0; q < PF; ++q) {
+      if (q < p.k) {
+        load_v(ring[q], Ab + (long long)q * p.lda, q, p.m, lane);
+        tr[q] = tg[q];
       }
+    }
+#pragma unroll 1
+    for (int i0 = 0; i0 < p.k; i0 += PF) {
 #pragma unroll
-      for (int s = 0; s < MR; ++s) v[s] = vn[s];
+      for (int q = 0; q < PF; ++q) {
+        const int i = i0 + q;
+        if (i < p.k) {
+          apply_one(b, ring[q], X::conj(tr[q]), i, p.m, lane);
+          if (i + PF < p.k) {
+            load_v(ring[q], Ab + (long long)(i + PF) * p.lda, i + PF, p.m, lane);
+            tr[q] = tg[i + PF];
+          }
+        }
+      }
     }
 #pragma unroll
     for (int s = 0; s < MR; ++s)
@@ -84,9 +118,9 @@ struct ApplyQh {
   }
 };
 
-template <class T, int MR, int NB>
-__global__ void __launch_bounds__(128) apply_qh_kernel(const ApplyArgs p) {
-  ApplyQh<T, MR, NB>::run(p);
+template <class T, int MR, int NB, int PF>
+__global__ void __launch_bounds__(ApplyQh<T, MR, NB, PF>::kWarps * 32) apply_qh_kernel(const ApplyArgs p) {
+  ApplyQh<T, MR, NB, PF>::run(p);
 }
 
 }  // namespace bqr
