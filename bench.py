@@ -167,6 +167,15 @@ class Workload:
         if st:
             raise RuntimeError(f"bqr_geqrf_batched -> {st}")
 
+    def geqrf_qhb(self):
+        """Fused factorisation + Q^H b (one kernel for the STAP shape)."""
+        c = self.c
+        st = self.lib.bqr_geqrf_qhb_batched(self.code, self.m, self.n, self.nrhs, self.batch,
+                                            c.c_void_p(self.A.data_ptr()), self.m, c.c_void_p(self.tau.data_ptr()),
+                                            c.c_void_p(self.B.data_ptr()), self.m, c.c_void_p(self.sptr))
+        if st:
+            raise RuntimeError(f"bqr_geqrf_qhb_batched -> {st}")
+
     def apply(self):
         c = self.c
         st = self.lib.bqr_apply_qh_batched(self.code, self.m, self.n, self.k, self.nrhs, self.batch,
@@ -184,27 +193,39 @@ def max_over_ranks(torch, dist, world, x: float) -> float:
     return bqr_dist.max_over_ranks(torch, dist, x)
 
 
-def time_workload(w: Workload, steps: int, warmup: int, torch, dist, world, flush, sampler=None):
-    """Returns (ms_per_step, ms_geqrf_per_launch)."""
+def time_workload(w: Workload, steps: int, warmup: int, torch, dist, world, flush, sampler=None, fused=True):
+    """Returns (ms_per_step, ms_of_the_factorisation_kernel).  With right-hand
+    sides the step is the fused factorisation + Q^H b (one kernel, the
+    augmented [A | b] of P:L313) unless fused=False (geqrf, then apply)."""
     ev = [[torch.cuda.Event(enable_timing=True) for _ in range(3)] for _ in range(steps)]
+
+    def run_step(i=None):
+        if i is not None:
+            ev[i][0].record(w.stream)
+        if w.nrhs and fused:
+            w.geqrf_qhb()
+            if i is not None:
+                ev[i][1].record(w.stream)
+        else:
+            w.geqrf()
+            if i is not None:
+                ev[i][1].record(w.stream)
+            if w.nrhs:
+                w.apply()
+        if i is not None:
+            ev[i][2].record(w.stream)
+
     for _ in range(warmup):
         w.restore()
         flush.zero_()
-        w.geqrf()
-        if w.nrhs:
-            w.apply()
+        run_step()
     barrier(torch, dist, world)
     ctx = sampler if sampler is not None else _Null()
     with ctx:
         for i in range(steps):
             w.restore()
             flush.zero_()
-            ev[i][0].record(w.stream)
-            w.geqrf()
-            ev[i][1].record(w.stream)
-            if w.nrhs:
-                w.apply()
-            ev[i][2].record(w.stream)
+            run_step(i)
         barrier(torch, dist, world)
     step_ms = sum(e[0].elapsed_time(e[2]) for e in ev) / steps
     qr_ms = sum(e[0].elapsed_time(e[1]) for e in ev) / steps
@@ -219,23 +240,28 @@ class _Null:
         pass
 
 
-def roofline_obj(w: Workload, qr_ms: float, peaks: dict, n_sm: int):
-    """Roofline of the dominant kernel (the geqrf launch): SURVEY 8(d)."""
+def roofline_obj(w: Workload, qr_ms: float, peaks: dict, n_sm: int, fused: bool = False):
+    """Roofline of the dominant kernel (the geqrf launch, or the fused
+    geqrf + Q^H b launch for configs with right-hand sides): SURVEY 8(d)."""
     hbm = float(peaks["hbm_gbs"])
     fp32 = bm.fp32_peak_tflops(n_sm, float(peaks.get("sm_max_mhz", 1965.0)))
-    t_roof, bound = bm.roofline_time_s(w.flops, w.bytes, hbm, fp32)
+    flops = w.flops + (w.flops_apply if fused else 0)
+    nbytes = w.bytes + (w.bytes_apply if fused else 0)
+    t_roof, bound = bm.roofline_time_s(flops, nbytes, hbm, fp32)
     t = qr_ms / 1e3
     traffic = load_traffic(w.name)
     if bound == "hbm":
-        ach, peak, unit = w.bytes / t / 1e9, hbm, "GB/s"
+        ach, peak, unit = nbytes / t / 1e9, hbm, "GB/s"
     else:
-        ach, peak, unit = w.flops / t / 1e12, fp32, "TFLOP/s"
+        ach, peak, unit = flops / t / 1e12, fp32, "TFLOP/s"
     return {"bound": bound, "achieved": round(ach, 3), "peak": peak, "unit": unit,
             "frac": round(ach / peak, 4), "traffic": traffic,
             "peak_source": ("MEASURED_PEAKS.json hbm_gbs" if bound == "hbm" else
                             f"derived: {n_sm} SMs x 128 FP32 lanes x 2 x {peaks.get('sm_max_mhz', 1965.0)} MHz"),
             "roofline_us": round(t_roof * 1e6, 3), "kernel_us": round(qr_ms * 1e3, 3),
-            "algorithmic_bytes": w.bytes, "useful_flops": w.flops}
+            "algorithmic_bytes": nbytes, "useful_flops": flops,
+            "kernel": (w.bqr.load().bqr_qhb_kernel_name(w.code, w.m, w.n, w.nrhs).decode() if fused
+                       else w.bqr.kernel_name(w.code, w.m, w.n))}
 
 
 def e2e_host(w: Workload, steps: int, warmup: int, torch, dist, world):
@@ -323,8 +349,8 @@ def run_ours(args):
         "vs_baseline": None, "dtype": "f32" if main.dt == "f32" else "c64", "data": "synthetic (seeded iid Gaussian, bqr_inputs)",
         "config": config_block(main, world, l2_note),
         "matrices_per_s": round(world * main.batch / (step_ms / 1e3), 1),
-        "roofline": roofline_obj(main, qr_ms, peaks, n_sm),
-        "gpu_launches": args.steps * (2 if main.nrhs else 1),
+        "roofline": roofline_obj(main, qr_ms, peaks, n_sm, fused=bool(main.nrhs)),
+        "gpu_launches": args.steps,
         "clocks": sampler.summary(),
     }
     # end to end through the public host-buffer API
@@ -346,10 +372,14 @@ def run_ours(args):
                           "ms_per_step": round(s_ms, 6), "steps": k2,
                           "matrices_per_s": round(world * w.batch / (s_ms / 1e3), 1),
                           "config": config_block(w, world, l2_note),
-                          "roofline": roofline_obj(w, q_ms, peaks, n_sm)}
+                          "roofline": roofline_obj(w, q_ms, peaks, n_sm, fused=bool(w.nrhs))}
+            out["gpu_launches"] += k2
             if w.nrhs:
-                also[name]["apply_ms"] = round(s_ms - q_ms, 6)
-            out["gpu_launches"] += k2 * (2 if w.nrhs else 1)
+                # context: the same step as two launches (geqrf, then apply_qh)
+                s2, q2 = time_workload(w, k2, max(3, args.warmup), torch, dist, world, flush, fused=False)
+                also[name]["unfused_two_launch"] = {"ms_per_step": round(s2, 6), "geqrf_ms": round(q2, 6),
+                                                    "apply_ms": round(s2 - q2, 6)}
+                out["gpu_launches"] += 2 * k2
             del w
         out["also"] = also
     # determinism evidence (outside the timed region): checksum of one

@@ -23,7 +23,7 @@ import os
 __all__ = [
     "load", "colmajor", "geqrf_batched", "orgqr_batched", "apply_qh_batched",
     "geqrf_batched_host", "host_workspace_bytes", "kernel_name", "geqrf_launches",
-    "BQRError", "R32", "C64", "lib_path", "geqrf_batched_ptr",
+    "BQRError", "R32", "C64", "lib_path", "geqrf_batched_ptr", "geqrf_qhb_batched",
 ]
 
 R32, C64 = 0, 1
@@ -54,6 +54,10 @@ def load():
     lib.bqr_geqrf_batched.argtypes = [i, i, i, i, p, i, p, p]
     lib.bqr_orgqr_batched.argtypes = [i, i, i, i, i, p, i, p, p]
     lib.bqr_apply_qh_batched.argtypes = [i, i, i, i, i, i, p, i, p, p, i, p]
+    lib.bqr_geqrf_qhb_batched.argtypes = [i, i, i, i, i, p, i, p, p, i, p]
+    lib.bqr_geqrf_qhb_batched.restype = i
+    lib.bqr_qhb_kernel_name.argtypes = [i, i, i, i]
+    lib.bqr_qhb_kernel_name.restype = ctypes.c_char_p
     lib.bqr_geqrf_batched_host.argtypes = [i, i, i, i, p, i, p, p, sz, p]
     lib.bqr_host_workspace_bytes.argtypes = [i, i, i, i, i]
     lib.bqr_host_workspace_bytes.restype = sz
@@ -161,6 +165,24 @@ def apply_qh_batched(A, tau, B, stream=None):
                                      _stream_ptr(stream))
     _check(st, "bqr_apply_qh_batched")
     return B
+
+
+def geqrf_qhb_batched(A, B, tau=None, stream=None):
+    """Fused: A <- [R; V] and B <- Q^H B in one kernel (the augmented [A | b]
+    of P:L313).  Returns (A, tau, B)."""
+    import torch
+    batch, m, n = A.shape
+    m, n, lda = _layout(A)
+    _, mb, nrhs = B.shape
+    _, _, ldb = _layout(B)
+    k = min(m, n)
+    if tau is None:
+        tau = torch.empty((batch, k), dtype=A.dtype, device=A.device)
+    st = load().bqr_geqrf_qhb_batched(_dtype_code(A), m, n, nrhs, batch, ctypes.c_void_p(A.data_ptr()), lda,
+                                      ctypes.c_void_p(tau.data_ptr()), ctypes.c_void_p(B.data_ptr()), ldb,
+                                      _stream_ptr(stream))
+    _check(st, "bqr_geqrf_qhb_batched")
+    return A, tau, B
 
 
 def host_workspace_bytes(dtype: int, m: int, n: int, lda: int, chunk: int) -> int:

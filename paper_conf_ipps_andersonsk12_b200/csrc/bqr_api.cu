@@ -59,6 +59,8 @@ struct Call {
   long long batch;
   int m, n, k, lda;
   cudaStream_t stream;
+  void *B = nullptr;  // fused Q^H B (augmented columns); direct-load classes only
+  int ldb = 1, nrhs = 0;
 };
 
 using LaunchFn = int (*)(const Call &);
@@ -78,6 +80,7 @@ template <class T, int R, int G, int MR, int NC, int GPB, bool STAGE, bool EX, b
 int launch_rf(const Call &c) {
   using Cfg = RfCfg<T, R, G, MR, NC, GPB, STAGE, EX>;
   if (EX && (c.m != R * MR || c.n != G * NC)) return BQR_ERR_NOT_SUPPORTED;
+  if (c.nrhs > 0 && (STAGE || EX || ORG || c.n + c.nrhs > G * NC)) return BQR_ERR_NOT_SUPPORTED;
   RfArgs a;
   a.A = c.A;
   a.tau = c.tau;
@@ -91,6 +94,9 @@ int launch_rf(const Call &c) {
   const bool aligned = (reinterpret_cast<uintptr_t>(c.A) & 15) == 0;
   a.vec4 = (STAGE && (c.lda % 4 == 0) && (c.m % 4 == 0) && aligned) ? 1 : 0;
   a.bulk = (STAGE && c.lda == c.m && a.ldS == c.m && aligned && ((size_t)c.m * c.n * sizeof(T)) % 16 == 0) ? 1 : 0;
+  a.B = c.B;
+  a.ldb = c.ldb;
+  a.nrhs = c.nrhs;
   const size_t smem = (size_t)Cfg::kSmallAll * 4 + (STAGE ? (size_t)GPB * a.tileWords * 4 : 0);
   auto kern = ORG ? orgqr_rf_kernel<T, R, G, MR, NC, GPB, STAGE, EX> : geqrf_rf_kernel<T, R, G, MR, NC, GPB, STAGE, EX>;
   if (!ensure_smem(kern, smem)) return BQR_ERR_CUDA;
@@ -140,6 +146,8 @@ const ClassEntry kClasses[] = {
     {BQR_R32, 56, 56, 56, 56, true, RF_PLAN(float, 2, 8, 28, 7, 2, true, "rf_f32_R2G8_28x7_x2_stage")},
     {BQR_C64, 240, 66, 240, 66, false, RF_PLAN(float2, 32, 11, 8, 6, 1, false, "rf_c64_R32G11_8x6_cta")},
     {BQR_C64, 240, 66, 240, 66, true, RF_PLAN(float2, 16, 22, 15, 3, 1, false, "rf_c64_R16G22_15x3_cta")},
+    // 240x66 with up to 6 augmented right-hand sides (fused Q^H B)
+    {BQR_C64, 256, 72, 240, 67, true, RF_PLAN(float2, 32, 12, 8, 6, 1, false, "rf_c64_R32G12_8x6_cta")},
     // alternatives kept for measurement (BQR_FORCE_VARIANT)
     {BQR_R32, 56, 56, 56, 56, true, RF_PLAN(float, 4, 8, 14, 7, 1, true, "rf_f32_R4G8_14x7_x1_stage")},
     {BQR_R32, 56, 56, 56, 56, true, RF_PLAN(float, 4, 4, 14, 14, 2, true, "rf_f32_R4G4_14x14_x2_stage")},
@@ -201,6 +209,20 @@ Plan tiny_plan(int m, int n) {
     case 8: return tiny_plan_n<T, 8>(n);
   }
   return Plan{nullptr, nullptr, nullptr};
+}
+
+// fused geqrf + Q^H B: first direct-load class whose tile holds n + nrhs
+// columns (the augmented matrix of P:L313)
+const Plan *pick_fused(bqr_dtype_t dt, int m, int n, int nrhs) {
+  const Plan *best = nullptr;
+  int best_area = 1 << 30;
+  for (const auto &e : kClasses) {
+    if (e.dt != dt || m > e.mmax || n + nrhs > e.nmax) continue;
+    if (std::strstr(e.plan.name, "stage") || std::strstr(e.plan.name, "exact")) continue;
+    const int area = e.mmax * e.nmax;
+    if (area < best_area) { best = &e.plan; best_area = area; }
+  }
+  return best;
 }
 
 // geqrf plan; tiny sizes get their own thread-per-matrix kernel.
@@ -293,6 +315,12 @@ const char *bqr_status_string(int status) {
   return "unknown status";
 }
 
+const char *bqr_qhb_kernel_name(bqr_dtype_t dtype, int m, int n, int nrhs) {
+  if (!valid_dtype(dtype) || m <= 0 || n <= 0 || m < n || nrhs <= 0) return "";
+  const Plan *p = pick_fused(dtype, m, n, nrhs);
+  return p ? p->name : "";
+}
+
 const char *bqr_kernel_name(bqr_dtype_t dtype, int m, int n) {
   if (!valid_dtype(dtype) || m <= 0 || n <= 0 || m < n) return "";
   Plan p;
@@ -324,6 +352,39 @@ int bqr_geqrf_batched(bqr_dtype_t dtype, int m, int n, int batch, void *A, int l
   if (!geqrf_plan(dtype, m, n, &p)) return BQR_ERR_NOT_SUPPORTED;
   Call c{A, tau, batch, m, n, std::min(m, n), lda, stream};
   return p.geqrf(c);
+}
+
+int bqr_geqrf_qhb_batched(bqr_dtype_t dtype, int m, int n, int nrhs, int batch, void *A, int lda, void *tau,
+                          void *B, int ldb, cudaStream_t stream) {
+  if (!valid_dtype(dtype)) return -1;
+  if (m < 0) return -2;
+  if (n < 0) return -3;
+  if (nrhs < 0) return -4;
+  if (batch < 0) return -5;
+  const bool work = m > 0 && n > 0 && batch > 0;
+  if (work && A == nullptr) return -6;
+  if (lda < std::max(1, m)) return -7;
+  if (work && tau == nullptr) return -8;
+  if (work && nrhs > 0 && B == nullptr) return -9;
+  if (ldb < std::max(1, m)) return -10;
+  if (!work) return BQR_SUCCESS;
+  if ((reinterpret_cast<uintptr_t>(A) | reinterpret_cast<uintptr_t>(tau) | reinterpret_cast<uintptr_t>(B)) %
+      elem_size(dtype))
+    return BQR_ERR_MISALIGNED;
+  if (m < n) return BQR_ERR_NOT_SUPPORTED;
+  const int k = std::min(m, n);
+  if (const Plan *p = (nrhs > 0) ? pick_fused(dtype, m, n, nrhs) : nullptr) {
+    Call c{A, tau, batch, m, n, k, lda, stream};
+    c.B = B;
+    c.ldb = ldb;
+    c.nrhs = nrhs;
+    const int st = p->geqrf(c);
+    if (st != BQR_ERR_NOT_SUPPORTED) return st;
+  }
+  // no class holds the augmented tile: factor, then apply (two launches)
+  int st = bqr_geqrf_batched(dtype, m, n, batch, A, lda, tau, stream);
+  if (st != BQR_SUCCESS || nrhs == 0) return st;
+  return bqr_apply_qh_batched(dtype, m, n, k, nrhs, batch, A, lda, tau, B, ldb, stream);
 }
 
 int bqr_orgqr_batched(bqr_dtype_t dtype, int m, int n, int k, int batch, void *A, int lda,

@@ -31,11 +31,21 @@ struct ApplyQh {
 
   // raw column (rows >= i); the v_i = 1 / zero-above masks are applied at
   // use time, so nothing consumes the load until the ring comes round
+  // (asm volatile: ptxas otherwise sinks the loads to their first use, which
+  // turns the prefetch ring back into one exposed memory latency per column)
+  static __device__ __forceinline__ void ldg(float &d, const float *p, bool pred) {
+    asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.b32 q, %2, 0;\n\t@q ld.global.nc.f32 %0, [%1];\n}"
+                 : "+f"(d) : "l"(p), "r"((int)pred));
+  }
+  static __device__ __forceinline__ void ldg(float2 &d, const float2 *p, bool pred) {
+    asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.b32 q, %3, 0;\n\t@q ld.global.nc.v2.f32 {%0, %1}, [%2];\n}"
+                 : "+f"(d.x), "+f"(d.y) : "l"(p), "r"((int)pred));
+  }
   static __device__ __forceinline__ void load_v(T (&v)[MR], const T *col, int i, int m, int lane) {
 #pragma unroll
     for (int s = 0; s < MR; ++s) {
       const int r = lane + 32 * s;
-      if (r >= i && r < m) v[s] = col[r];
+      ldg(v[s], col + r, r >= i && r < m);
     }
   }
 
@@ -103,7 +113,7 @@ struct ApplyQh {
           apply_one(b, ring[q], X::conj(tr[q]), i, p.m, lane);
           if (i + PF < p.k) {
             load_v(ring[q], Ab + (long long)(i + PF) * p.lda, i + PF, p.m, lane);
-            tr[q] = tg[i + PF];
+            ldg(tr[q], tg + i + PF, true);
           }
         }
       }

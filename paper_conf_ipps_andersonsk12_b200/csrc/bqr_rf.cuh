@@ -45,6 +45,12 @@ struct RfArgs {
   int vec4;       // 16-byte vectorised staging legal (lda%4==0, m%4==0, aligned)
   int bulk;       // contiguous matrices (lda == m), 16-byte aligned, size % 16 == 0:
                   // stage with one TMA bulk copy per matrix each way
+  // augmented right-hand sides (the paper's [A | b]): columns
+  // n .. n+nrhs-1 of the register tile are B; they are updated by every
+  // reflector but never become pivots, so they end as Q^H B.  Direct
+  // (non-staged) kernels only; nrhs = 0 otherwise.
+  void *B;
+  int ldb, nrhs;
 };
 
 // Warp barrier as opaque PTX: nvcc versions the whole rest of a kernel on
@@ -200,6 +206,7 @@ struct RfKernel {
     T *taus;   // [NMAX]
     int rg, cg, t, lane, grp;
     int wid;   // warp index in the group, warp-uniform by construction (shfl)
+    long long mat;
     int kmax;
   };
 
@@ -649,6 +656,8 @@ struct RfKernel {
   }
 
   // ------------------------------------------------------------ staging
+  static __device__ __forceinline__ long long c_mat(const Ctx &c) { return c.mat; }
+
   // in-bounds test; compile-time true for exact-shape instantiations
   static __device__ __forceinline__ bool inb(int r, int col, int m, int n) {
     if constexpr (EX) return true;
@@ -707,12 +716,16 @@ struct RfKernel {
           a[i][j] = (inb(r, col, m, n) && (EX || active)) ? tile[r + col * ld] : 0.f;
         }
     } else {
+      const T *Bb = reinterpret_cast<const T *>(p.B) + c_mat(c) * (long long)p.ldb * p.nrhs;
 #pragma unroll
       for (int i = 0; i < MR; ++i)
 #pragma unroll
         for (int j = 0; j < NC; ++j) {
           const int r = c.rg + R * i, col = c.cg + G * j;
-          a[i][j] = (active && inb(r, col, m, n)) ? Ab[r + (long long)col * p.lda] : X::zero();
+          T x = X::zero();
+          if (active && inb(r, col, m, n)) x = Ab[r + (long long)col * p.lda];
+          if (!EX && active && r < m && col >= n && col < n + p.nrhs) x = Bb[r + (long long)(col - n) * p.ldb];
+          a[i][j] = x;
         }
     }
   }
@@ -763,12 +776,14 @@ struct RfKernel {
         }
       }
     } else if (active) {
+      T *Bb = reinterpret_cast<T *>(p.B) + c_mat(c) * (long long)p.ldb * p.nrhs;
 #pragma unroll
       for (int i = 0; i < MR; ++i)
 #pragma unroll
         for (int j = 0; j < NC; ++j) {
           const int r = c.rg + R * i, col = c.cg + G * j;
           if (inb(r, col, m, n)) Ab[r + (long long)col * p.lda] = a[i][j];
+          if (!EX && r < m && col >= n && col < n + p.nrhs) Bb[r + (long long)(col - n) * p.ldb] = a[i][j];
         }
     }
   }
@@ -790,6 +805,7 @@ struct RfKernel {
     long long mat = (long long)blockIdx.x * GPB + grp;
     const bool active = mat < p.batch;
     if (!active) mat = p.batch - 1;
+    c.mat = mat;
     float *gs = smem + grp * Cfg::kSmallWords;
     c.vbuf = reinterpret_cast<T *>(gs);
     c.taus = c.vbuf + NBUF * VB;

@@ -56,3 +56,19 @@ def apply_gpu(RV_cm: np.ndarray, m: int, k: int, tau: np.ndarray, B_cm: np.ndarr
     assert st == 0
     torch.cuda.synchronize()
     return B.cpu().numpy()
+
+
+def geqrf_qhb_gpu(A_cm: np.ndarray, m: int, B_cm: np.ndarray):
+    """Fused geqrf + Q^H B through bqr_geqrf_qhb_batched."""
+    import ctypes
+    A = to_dev(A_cm)
+    B = to_dev(B_cm)
+    batch, n, lda = A_cm.shape
+    _, nrhs, ldb = B_cm.shape
+    tau = torch.empty((batch, min(m, n)), dtype=A.dtype, device="cuda")
+    st = bqr.load().bqr_geqrf_qhb_batched(bqr.R32 if A.dtype == torch.float32 else bqr.C64, m, n, nrhs, batch,
+                                          ctypes.c_void_p(A.data_ptr()), lda, ctypes.c_void_p(tau.data_ptr()),
+                                          ctypes.c_void_p(B.data_ptr()), ldb, None)
+    assert st == 0, st
+    torch.cuda.synchronize()
+    return A.cpu().numpy(), tau.cpu().numpy(), B.cpu().numpy()

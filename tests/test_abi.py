@@ -127,3 +127,16 @@ def test_no_fallback_when_library_missing(monkeypatch, tmp_path):
     with pytest.raises(mod.BQRError):
         mod.load()
     importlib.reload(bqr)
+
+
+@pytest.mark.parametrize("args,code", [
+    ((0, 8, 4, -1, 1, FAKE, 8, FAKE, FAKE, 8), -4),
+    ((0, 8, 4, 1, 1, FAKE, 8, FAKE, 0, 8), -9),
+    ((0, 8, 4, 1, 1, FAKE, 8, FAKE, FAKE, 7), -10),
+    ((0, 8, 4, 1, 0, 0, 8, 0, 0, 8), 0),
+])
+def test_qhb_argument_checks(lib, args, code):
+    d, m, n, nrhs, b, A, lda, tau, B, ldb = args
+    st = lib.bqr_geqrf_qhb_batched(d, m, n, nrhs, b, ctypes.c_void_p(A), lda, ctypes.c_void_p(tau),
+                                   ctypes.c_void_p(B), ldb, None)
+    assert st == code

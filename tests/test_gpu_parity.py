@@ -15,7 +15,7 @@ pytestmark = pytest.mark.gpu
 if not torch.cuda.is_available():  # pragma: no cover
     pytest.skip("needs a GPU", allow_module_level=True)
 
-from gpu_util import apply_gpu, geqrf_gpu, orgqr_gpu  # noqa: E402
+from gpu_util import apply_gpu, geqrf_gpu, geqrf_qhb_gpu, orgqr_gpu  # noqa: E402
 
 
 def _check(A, m, full_q=True):
@@ -190,3 +190,23 @@ def test_host_buffer_api():
     bqr.geqrf_batched_host(bqr.R32, 56, 56, 1000, Ah.data_ptr(), 56, tau_h.data_ptr(), ws.data_ptr(), wsb)
     assert np.array_equal(Ah.numpy().view(np.uint32), dev_out.view(np.uint32))
     assert np.array_equal(tau_h.numpy().view(np.uint32), dev_tau.view(np.uint32))
+
+
+@pytest.mark.parametrize("dt,m,n,nrhs", [("c64", 240, 66, 1), ("c64", 240, 66, 4), ("c64", 80, 16, 2),
+                                         ("f32", 100, 30, 3), ("f32", 56, 56, 1), ("c64", 8, 8, 1)])
+def test_fused_geqrf_qhb(dt, m, n, nrhs):
+    """The augmented [A | B] factorisation: R/V/tau pass the geqrf
+    comparator and B matches the oracle's Q^H B built from the GPU's own
+    reflectors (one kernel when a size class holds n + nrhs columns)."""
+    A = bqr_inputs.random_batch(m, n, 40, dt, seed=91)
+    B = bqr_inputs.rhs_batch(m, nrhs, 40, dt, seed=91)
+    out, tau, QhB = geqrf_qhb_gpu(A, m, B)
+    rep = compare_geqrf(A, m, out, tau, full_q=m <= 128)
+    assert rep["ok"], rep
+    r = compare_apply(out, m, min(m, n), tau, B, QhB)
+    assert r["ok"], r
+
+
+def test_fused_stap_is_one_kernel():
+    import paper_conf_ipps_andersonsk12_b200 as bqr
+    assert bqr.load().bqr_qhb_kernel_name(bqr.C64, 240, 66, 1).decode().startswith("rf_c64")
