@@ -61,6 +61,7 @@ struct Call {
   cudaStream_t stream;
   void *B = nullptr;  // fused Q^H B (augmented columns); direct-load classes only
   int ldb = 1, nrhs = 0;
+  long long strideA = -1, strideT = -1;  // batch strides; -1 = LAPACK-contiguous
 };
 
 using LaunchFn = int (*)(const Call &);
@@ -97,6 +98,10 @@ int launch_rf(const Call &c) {
   a.B = c.B;
   a.ldb = c.ldb;
   a.nrhs = c.nrhs;
+  a.strideA = c.strideA >= 0 ? c.strideA : (long long)c.lda * c.n;
+  a.strideT = c.strideT >= 0 ? c.strideT : (long long)c.k;
+  a.strideB = (long long)c.ldb * c.nrhs;
+  if (c.strideA >= 0) a.bulk = 0;  // panel views are not contiguous matrices
   const size_t smem = (size_t)Cfg::kSmallAll * 4 + (STAGE ? (size_t)GPB * a.tileWords * 4 : 0);
   auto kern = ORG ? orgqr_rf_kernel<T, R, G, MR, NC, GPB, STAGE, EX> : geqrf_rf_kernel<T, R, G, MR, NC, GPB, STAGE, EX>;
   if (!ensure_smem(kern, smem)) return BQR_ERR_CUDA;
@@ -225,6 +230,51 @@ const Plan *pick_fused(bqr_dtype_t dt, int m, int n, int nrhs) {
   return best;
 }
 
+// Oversize shapes (no single-SM class holds m x n; paper Sec. VII: "a
+// sequential tiled QR factorization algorithm similar to the approach in
+// the PLASMA library"): right-looking panels of width nb, each
+// factored by the register-file kernel of the tall-skinny class and applied
+// to the trailing columns by the Q^H B kernel, on panel views of the batch
+// (custom batch strides; 2 launches per panel).
+bool tiled_panel_width(bqr_dtype_t dt, int m, int n, int *nb) {
+  if (m > 256) return false;
+  *nb = dt == BQR_R32 ? 64 : 96;  // widest tall class: fp32 256x64, c64 256x96
+  return n > *nb;
+}
+
+template <class T>
+int launch_apply_views(const void *A, int lda, long long sA, const void *tau, long long sT, void *B, int ldb,
+                       long long sB, int m, int k, int nrhs, long long batch, cudaStream_t s);
+
+int geqrf_tiled(bqr_dtype_t dt, int m, int n, long long batch, void *A, int lda, void *tau, int nb,
+                cudaStream_t stream) {
+  const int kmax = std::min(m, n);
+  const size_t es = dt == BQR_R32 ? 4 : 8;
+  const long long sA = (long long)lda * n;
+  char *Ab = reinterpret_cast<char *>(A);
+  char *tb = reinterpret_cast<char *>(tau);
+  for (int k0 = 0; k0 < kmax; k0 += nb) {
+    const int w = std::min(nb, kmax - k0), mp = m - k0;
+    const Plan *p = pick(dt, mp, w);
+    if (!p) return BQR_ERR_NOT_SUPPORTED;
+    Call c{Ab + (k0 + (size_t)k0 * lda) * es, tb + (size_t)k0 * es, batch, mp, w, std::min(mp, w), lda, stream};
+    c.strideA = sA;
+    c.strideT = kmax;
+    int st = p->geqrf(c);
+    if (st != BQR_SUCCESS) return st;
+    const int nrest = n - k0 - w;
+    if (nrest > 0) {
+      void *Bv = Ab + (k0 + (size_t)(k0 + w) * lda) * es;
+      st = dt == BQR_R32
+               ? launch_apply_views<float>(c.A, lda, sA, c.tau, kmax, Bv, lda, sA, mp, std::min(mp, w), nrest, batch, stream)
+               : launch_apply_views<float2>(c.A, lda, sA, c.tau, kmax, Bv, lda, sA, mp, std::min(mp, w), nrest, batch,
+                                            stream);
+      if (st != BQR_SUCCESS) return st;
+    }
+  }
+  return BQR_SUCCESS;
+}
+
 // geqrf plan; tiny sizes get their own thread-per-matrix kernel.
 bool geqrf_plan(bqr_dtype_t dt, int m, int n, Plan *out) {
   if (m <= 8 && n <= m && !forced_variant()) {
@@ -295,6 +345,13 @@ __global__ void selftest_math_kernel(long long n, unsigned seed, unsigned long l
   atomicAdd(&counts[2], bad_rcp);
 }
 
+template <class T>
+int launch_apply_views(const void *A, int lda, long long sA, const void *tau, long long sT, void *B, int ldb,
+                       long long sB, int m, int k, int nrhs, long long batch, cudaStream_t s) {
+  ApplyArgs a{A, tau, B, batch, lda, 0, m, k, nrhs, ldb, sA, sT, sB};
+  return apply_dispatch<T>(a, s);
+}
+
 bool valid_dtype(int d) { return d == BQR_R32 || d == BQR_C64; }
 size_t elem_size(bqr_dtype_t d) { return d == BQR_R32 ? 4 : 8; }
 
@@ -324,14 +381,24 @@ const char *bqr_qhb_kernel_name(bqr_dtype_t dtype, int m, int n, int nrhs) {
 const char *bqr_kernel_name(bqr_dtype_t dtype, int m, int n) {
   if (!valid_dtype(dtype) || m <= 0 || n <= 0 || m < n) return "";
   Plan p;
-  if (!geqrf_plan(dtype, m, n, &p)) return "";
+  if (!geqrf_plan(dtype, m, n, &p)) {
+    int nb;
+    return tiled_panel_width(dtype, m, n, &nb) ? (dtype == BQR_R32 ? "tiled_f32_panel64+apply" : "tiled_c64_panel96+apply")
+                                                : "";
+  }
   return p.name ? p.name : "";
 }
 
 int bqr_geqrf_launches(bqr_dtype_t dtype, int m, int n, int batch) {
-  if (!valid_dtype(dtype) || m <= 0 || n <= 0 || batch <= 0) return 0;
+  if (!valid_dtype(dtype) || m <= 0 || n <= 0 || batch <= 0 || m < n) return 0;
   Plan p;
-  return geqrf_plan(dtype, m, n, &p) ? 1 : 0;
+  if (geqrf_plan(dtype, m, n, &p)) return 1;
+  int nb;
+  if (!tiled_panel_width(dtype, m, n, &nb)) return 0;
+  int launches = 0;
+  const int kmax = std::min(m, n);
+  for (int k0 = 0; k0 < kmax; k0 += nb) launches += (n - k0 - std::min(nb, kmax - k0) > 0) ? 2 : 1;
+  return launches;
 }
 
 int bqr_geqrf_batched(bqr_dtype_t dtype, int m, int n, int batch, void *A, int lda, void *tau,
@@ -349,7 +416,11 @@ int bqr_geqrf_batched(bqr_dtype_t dtype, int m, int n, int batch, void *A, int l
     return BQR_ERR_MISALIGNED;
   if (m < n) return BQR_ERR_NOT_SUPPORTED;
   Plan p;
-  if (!geqrf_plan(dtype, m, n, &p)) return BQR_ERR_NOT_SUPPORTED;
+  if (!geqrf_plan(dtype, m, n, &p)) {
+    int nb;
+    if (tiled_panel_width(dtype, m, n, &nb)) return geqrf_tiled(dtype, m, n, batch, A, lda, tau, nb, stream);
+    return BQR_ERR_NOT_SUPPORTED;
+  }
   Call c{A, tau, batch, m, n, std::min(m, n), lda, stream};
   return p.geqrf(c);
 }
@@ -425,7 +496,7 @@ int bqr_apply_qh_batched(bqr_dtype_t dtype, int m, int n, int k, int nrhs, int b
   if ((reinterpret_cast<uintptr_t>(A) | reinterpret_cast<uintptr_t>(tau) |
        reinterpret_cast<uintptr_t>(B)) % elem_size(dtype))
     return BQR_ERR_MISALIGNED;
-  ApplyArgs a{A, tau, B, batch, lda, n, m, k, nrhs, ldb};
+  ApplyArgs a{A, tau, B, batch, lda, n, m, k, nrhs, ldb, (long long)lda * n, (long long)k, (long long)ldb * nrhs};
   return dtype == BQR_R32 ? apply_dispatch<float>(a, stream) : apply_dispatch<float2>(a, stream);
 }
 

@@ -22,6 +22,7 @@ struct ApplyArgs {
   void *B;
   long long batch;
   int lda, ncolsA, m, k, nrhs, ldb;
+  long long strideA, strideT, strideB;  // batch strides (elements)
 };
 
 template <class T, int MR, int NB, int PF>
@@ -78,9 +79,9 @@ struct ApplyQh {
     if (item >= p.batch * nblk) return;
     const long long mat = item / nblk;
     const int j0 = (int)(item - mat * nblk) * NB;
-    const T *Ab = reinterpret_cast<const T *>(p.A) + mat * (long long)p.lda * p.ncolsA;
-    const T *tg = reinterpret_cast<const T *>(p.tau) + mat * (long long)p.k;
-    T *Bb = reinterpret_cast<T *>(p.B) + mat * (long long)p.ldb * p.nrhs;
+    const T *Ab = reinterpret_cast<const T *>(p.A) + mat * p.strideA;
+    const T *tg = reinterpret_cast<const T *>(p.tau) + mat * p.strideT;
+    T *Bb = reinterpret_cast<T *>(p.B) + mat * p.strideB;
     T b[MR][NB];
 #pragma unroll
     for (int s = 0; s < MR; ++s)

@@ -51,6 +51,9 @@ struct RfArgs {
   // (non-staged) kernels only; nrhs = 0 otherwise.
   void *B;
   int ldb, nrhs;
+  // batch strides in elements (A, tau, B); LAPACK-contiguous batches use
+  // lda*n, kmax, ldb*nrhs; the tiled oversize path passes panel views
+  long long strideA, strideT, strideB;
 };
 
 // Warp barrier as opaque PTX: nvcc versions the whole rest of a kernel on
@@ -716,7 +719,7 @@ struct RfKernel {
           a[i][j] = (inb(r, col, m, n) && (EX || active)) ? tile[r + col * ld] : 0.f;
         }
     } else {
-      const T *Bb = reinterpret_cast<const T *>(p.B) + c_mat(c) * (long long)p.ldb * p.nrhs;
+      const T *Bb = reinterpret_cast<const T *>(p.B) + c_mat(c) * p.strideB;
 #pragma unroll
       for (int i = 0; i < MR; ++i)
 #pragma unroll
@@ -776,7 +779,7 @@ struct RfKernel {
         }
       }
     } else if (active) {
-      T *Bb = reinterpret_cast<T *>(p.B) + c_mat(c) * (long long)p.ldb * p.nrhs;
+      T *Bb = reinterpret_cast<T *>(p.B) + c_mat(c) * p.strideB;
 #pragma unroll
       for (int i = 0; i < MR; ++i)
 #pragma unroll
@@ -809,7 +812,7 @@ struct RfKernel {
     float *gs = smem + grp * Cfg::kSmallWords;
     c.vbuf = reinterpret_cast<T *>(gs);
     c.taus = c.vbuf + NBUF * VB;
-    T *Ab = reinterpret_cast<T *>(p.A) + mat * (long long)p.lda * p.n;
+    T *Ab = reinterpret_cast<T *>(p.A) + mat * p.strideA;
     T a[MR][NC];
     load_matrix(p, c, smem, Ab, active, a);
 
@@ -822,7 +825,7 @@ struct RfKernel {
           const int r = c.rg + R * i, col = c.cg + G * j;
           if (col >= p.kmax) a[i][j] = X::sel(r == col, X::one(), X::zero());
         }
-      const T *tg = reinterpret_cast<const T *>(p.tau) + mat * (long long)p.kmax;
+      const T *tg = reinterpret_cast<const T *>(p.tau) + mat * p.strideT;
       org_panels<NC - 1>(c, a, p.kmax, tg);
     } else {
       if constexpr (kFullUnroll && EX && GT <= 32) {
@@ -836,7 +839,7 @@ struct RfKernel {
     store_matrix(p, c, smem, Ab, active, a);
     // tau list -> global (each tau was published before a group barrier)
     if (!ORG && active) {
-      T *tg = reinterpret_cast<T *>(p.tau) + mat * (long long)p.kmax;
+      T *tg = reinterpret_cast<T *>(p.tau) + mat * p.strideT;
       for (int idx = t; idx < p.kmax; idx += GT) tg[idx] = c.taus[idx];
     }
   }

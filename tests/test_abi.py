@@ -113,6 +113,13 @@ def test_dispatch(lib, dt, m, n, expect):
     assert bqr.geqrf_launches(dt, m, n, 10) == 1
 
 
+@pytest.mark.parametrize("dt,n,launches", [(0, 256, 7), (0, 160, 5), (1, 256, 5), (1, 192, 3)])
+def test_tiled_dispatch(lib, dt, n, launches):
+    """Shapes above every single-SM class run as tiled panels."""
+    assert bqr.kernel_name(dt, n, n).startswith("tiled")
+    assert bqr.geqrf_launches(dt, n, n, 10) == launches
+
+
 def test_workspace_size(lib):
     w = bqr.host_workspace_bytes(0, 56, 56, 56, 100)
     assert w >= 2 * 100 * (56 * 56 + 56) * 4
