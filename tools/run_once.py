@@ -19,8 +19,9 @@ flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
 for _ in range(reps):
     w.restore()
     flush.zero_()
-    w.geqrf()
     if w.nrhs:
-        w.apply()
+        w.geqrf_qhb()  # the bench step: fused factorisation + Q^H b
+    else:
+        w.geqrf()
 torch.cuda.synchronize()
 print("done", name, bqr.kernel_name(w.code, w.m, w.n))
