@@ -27,10 +27,12 @@ rep = compare_geqrf(A, c['m'], out, tau, full_q=c['m'] <= 128)
 w = bench.Workload({cfg!r}, 0, 1, torch, bqr)
 flush = torch.empty(256 << 20, dtype=torch.uint8, device='cuda')
 class A_: pass
-s_ms, q_ms = bench.time_workload(w, 50, 5, torch, None, 1, flush)
+smp = bench.ClockSampler(0, 0.005)
+s_ms, q_ms = bench.time_workload(w, 50, 5, torch, None, 1, flush, sampler=smp, fused=False)
+clk = smp.summary()
 print(json.dumps({{'variant': {nm!r}, 'kernel': bqr.kernel_name(w.code, w.m, w.n), 'qr_us': round(q_ms*1e3, 2),
    'step_us': round(s_ms*1e3, 2), 'gflops': round(w.flops/(q_ms/1e3)/1e9, 1), 'parity_ok': rep['ok'],
-   'resid': rep['residual_max'], 'orth': rep['orth_max']}}))
+   'resid': rep['residual_max'], 'orth': rep['orth_max'], 'sm_mhz': clk['sm_mhz'], 'reasons': clk['reasons']}}))
 """
     r = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True)
     print(r.stdout.strip() or r.stderr[-2000:], flush=True)
