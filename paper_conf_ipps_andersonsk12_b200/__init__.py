@@ -54,10 +54,11 @@ def load():
     lib.bqr_geqrf_batched.argtypes = [i, i, i, i, p, i, p, p]
     lib.bqr_orgqr_batched.argtypes = [i, i, i, i, i, p, i, p, p]
     lib.bqr_apply_qh_batched.argtypes = [i, i, i, i, i, i, p, i, p, p, i, p]
-    lib.bqr_geqrf_qhb_batched.argtypes = [i, i, i, i, i, p, i, p, p, i, p]
-    lib.bqr_geqrf_qhb_batched.restype = i
-    lib.bqr_qhb_kernel_name.argtypes = [i, i, i, i]
-    lib.bqr_qhb_kernel_name.restype = ctypes.c_char_p
+    if hasattr(lib, "bqr_geqrf_qhb_batched"):  # absent in pre-fusion builds (A/B timing)
+        lib.bqr_geqrf_qhb_batched.argtypes = [i, i, i, i, i, p, i, p, p, i, p]
+        lib.bqr_geqrf_qhb_batched.restype = i
+        lib.bqr_qhb_kernel_name.argtypes = [i, i, i, i]
+        lib.bqr_qhb_kernel_name.restype = ctypes.c_char_p
     lib.bqr_geqrf_batched_host.argtypes = [i, i, i, i, p, i, p, p, sz, p]
     lib.bqr_host_workspace_bytes.argtypes = [i, i, i, i, i]
     lib.bqr_host_workspace_bytes.restype = sz

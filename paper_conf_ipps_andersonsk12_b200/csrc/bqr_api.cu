@@ -77,11 +77,11 @@ inline int staging_ld(int m) {
   return (m + 3) & ~3;
 }
 
-template <class T, int R, int G, int MR, int NC, int GPB, bool STAGE, bool EX, bool ORG>
+template <class T, int R, int G, int MR, int NC, int GPB, bool STAGE, bool EX, bool AUG, bool ORG>
 int launch_rf(const Call &c) {
   using Cfg = RfCfg<T, R, G, MR, NC, GPB, STAGE, EX>;
   if (EX && (c.m != R * MR || c.n != G * NC)) return BQR_ERR_NOT_SUPPORTED;
-  if (c.nrhs > 0 && (STAGE || EX || ORG || c.n + c.nrhs > G * NC)) return BQR_ERR_NOT_SUPPORTED;
+  if (c.nrhs > 0 && (!AUG || STAGE || EX || ORG || c.n + c.nrhs > G * NC)) return BQR_ERR_NOT_SUPPORTED;
   RfArgs a;
   a.A = c.A;
   a.tau = c.tau;
@@ -103,7 +103,7 @@ int launch_rf(const Call &c) {
   a.strideB = (long long)c.ldb * c.nrhs;
   if (c.strideA >= 0) a.bulk = 0;  // panel views are not contiguous matrices
   const size_t smem = (size_t)Cfg::kSmallAll * 4 + (STAGE ? (size_t)GPB * a.tileWords * 4 : 0);
-  auto kern = ORG ? orgqr_rf_kernel<T, R, G, MR, NC, GPB, STAGE, EX> : geqrf_rf_kernel<T, R, G, MR, NC, GPB, STAGE, EX>;
+  auto kern = ORG ? orgqr_rf_kernel<T, R, G, MR, NC, GPB, STAGE, EX, AUG> : geqrf_rf_kernel<T, R, G, MR, NC, GPB, STAGE, EX, AUG>;
   if (!ensure_smem(kern, smem)) return BQR_ERR_CUDA;
   const long long grid = (c.batch + GPB - 1) / GPB;
   if (grid > 0x7fffffffLL) return BQR_ERR_NOT_SUPPORTED;
@@ -128,12 +128,15 @@ int launch_tiny(const Call &c) {
 }
 
 // ---- size classes: smallest class that holds (m, n)
-#define RF_PLAN_X(T, R, G, MR, NC, GPB, STAGE, EX, NAME)                  \
+#define RF_PLAN_XA(T, R, G, MR, NC, GPB, STAGE, EX, AUG, NAME)             \
   Plan {                                                                 \
-    NAME, &launch_rf<T, R, G, MR, NC, GPB, STAGE, EX, false>,            \
-        &launch_rf<T, R, G, MR, NC, GPB, STAGE, EX, true>                \
+    NAME, &launch_rf<T, R, G, MR, NC, GPB, STAGE, EX, AUG, false>,       \
+        &launch_rf<T, R, G, MR, NC, GPB, STAGE, EX, false, true>         \
   }
+#define RF_PLAN_X(T, R, G, MR, NC, GPB, STAGE, EX, NAME) RF_PLAN_XA(T, R, G, MR, NC, GPB, STAGE, EX, false, NAME)
 #define RF_PLAN(T, R, G, MR, NC, GPB, STAGE, NAME) RF_PLAN_X(T, R, G, MR, NC, GPB, STAGE, false, NAME)
+// augmented (fused Q^H B) variant of a direct-load class
+#define RF_PLAN_AUG(T, R, G, MR, NC, NAME) RF_PLAN_XA(T, R, G, MR, NC, 1, false, false, true, NAME)
 
 struct ClassEntry {
   bqr_dtype_t dt;
@@ -151,8 +154,12 @@ const ClassEntry kClasses[] = {
     {BQR_R32, 56, 56, 56, 56, true, RF_PLAN(float, 2, 8, 28, 7, 2, true, "rf_f32_R2G8_28x7_x2_stage")},
     {BQR_C64, 240, 66, 240, 66, false, RF_PLAN(float2, 32, 11, 8, 6, 1, false, "rf_c64_R32G11_8x6_cta")},
     {BQR_C64, 240, 66, 240, 66, true, RF_PLAN(float2, 16, 22, 15, 3, 1, false, "rf_c64_R16G22_15x3_cta")},
+    {BQR_C64, 256, 72, 240, 66, true, RF_PLAN(float2, 32, 8, 8, 9, 1, false, "rf_c64_R32G8_8x9_cta")},
+    {BQR_C64, 240, 80, 240, 66, true, RF_PLAN(float2, 16, 16, 15, 5, 1, false, "rf_c64_R16G16_15x5_cta")},
     // 240x66 with up to 6 augmented right-hand sides (fused Q^H B)
-    {BQR_C64, 256, 72, 240, 67, true, RF_PLAN(float2, 32, 12, 8, 6, 1, false, "rf_c64_R32G12_8x6_cta")},
+    {BQR_C64, 256, 72, 240, 67, true, RF_PLAN_AUG(float2, 32, 12, 8, 6, "rf_c64_R32G12_8x6_aug")},
+    {BQR_C64, 128, 128, 0, 0, true, RF_PLAN_AUG(float2, 32, 16, 4, 8, "rf_c64_R32G16_4x8_aug")},
+    {BQR_R32, 128, 128, 0, 0, true, RF_PLAN_AUG(float, 32, 8, 4, 16, "rf_f32_R32G8_4x16_aug")},
     // alternatives kept for measurement (BQR_FORCE_VARIANT)
     {BQR_R32, 56, 56, 56, 56, true, RF_PLAN(float, 4, 8, 14, 7, 1, true, "rf_f32_R4G8_14x7_x1_stage")},
     {BQR_R32, 56, 56, 56, 56, true, RF_PLAN(float, 4, 4, 14, 14, 2, true, "rf_f32_R4G4_14x14_x2_stage")},
@@ -223,7 +230,7 @@ const Plan *pick_fused(bqr_dtype_t dt, int m, int n, int nrhs) {
   int best_area = 1 << 30;
   for (const auto &e : kClasses) {
     if (e.dt != dt || m > e.mmax || n + nrhs > e.nmax) continue;
-    if (std::strstr(e.plan.name, "stage") || std::strstr(e.plan.name, "exact")) continue;
+    if (!std::strstr(e.plan.name, "_aug")) continue;
     const int area = e.mmax * e.nmax;
     if (area < best_area) { best = &e.plan; best_area = area; }
   }

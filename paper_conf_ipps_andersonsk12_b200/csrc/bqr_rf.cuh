@@ -188,7 +188,7 @@ struct RfCfg {
   static constexpr int NMASK = (G % R == 0) ? G / R : (G + R - 1) / R + 1;
 };
 
-template <class T, int R, int G, int MR, int NC, int GPB, bool STAGE, bool EX = false>
+template <class T, int R, int G, int MR, int NC, int GPB, bool STAGE, bool EX = false, bool AUG = false>
 struct RfKernel {
   using Cfg = RfCfg<T, R, G, MR, NC, GPB, STAGE, EX>;
   using X = El<T>;
@@ -209,7 +209,6 @@ struct RfKernel {
     T *taus;   // [NMAX]
     int rg, cg, t, lane, grp;
     int wid;   // warp index in the group, warp-uniform by construction (shfl)
-    long long mat;
     int kmax;
   };
 
@@ -660,7 +659,12 @@ struct RfKernel {
   }
 
   // ------------------------------------------------------------ staging
-  static __device__ __forceinline__ long long c_mat(const Ctx &c) { return c.mat; }
+  // matrix index of this group (recomputed where needed: keeping it in the
+  // context costs two registers through the whole factorisation)
+  static __device__ __forceinline__ long long c_mat(const RfArgs &p, const Ctx &c) {
+    const long long mat = (long long)blockIdx.x * GPB + c.grp;
+    return mat < p.batch ? mat : p.batch - 1;
+  }
 
   // in-bounds test; compile-time true for exact-shape instantiations
   static __device__ __forceinline__ bool inb(int r, int col, int m, int n) {
@@ -720,7 +724,7 @@ struct RfKernel {
           a[i][j] = (inb(r, col, m, n) && (EX || active)) ? tile[r + col * ld] : 0.f;
         }
     } else {
-      const T *Bb = reinterpret_cast<const T *>(p.B) + c_mat(c) * p.strideB;
+      const T *Bb = reinterpret_cast<const T *>(p.B) + c_mat(p, c) * p.strideB;
 #pragma unroll
       for (int i = 0; i < MR; ++i)
 #pragma unroll
@@ -728,15 +732,23 @@ struct RfKernel {
           const int r = c.rg + R * i, col = c.cg + G * j;
           T x = X::zero();
           if (active && inb(r, col, m, n)) x = Ab[r + (long long)col * p.lda];
-          if (!EX && active && r < m && col >= n && col < n + p.nrhs) x = Bb[r + (long long)(col - n) * p.ldb];
+          if (AUG && active && r < m && col >= n && col < n + p.nrhs) x = Bb[r + (long long)(col - n) * p.ldb];
           a[i][j] = x;
         }
     }
   }
 
+  static __device__ __forceinline__ int opaque(int x) {
+    asm volatile("mov.b32 %0, %0;" : "+r"(x));
+    return x;
+  }
+
   static __device__ __forceinline__ void store_matrix(const RfArgs &p, Ctx &c, float *smem, T *Ab, bool active,
                                                       const T (&a)[MR][NC]) {
-    const int m = p.m, n = p.n;
+    // opaque reads: keeps ptxas from hoisting the store's per-element
+    // predicates above the factorisation loop (they would stay live in
+    // registers through it)
+    const int m = opaque(p.m), n = opaque(p.n);
     if constexpr (STAGE) {
       float *tile = smem + Cfg::kSmallAll + c.grp * p.tileWords;
       float *Ag = reinterpret_cast<float *>(Ab);
@@ -780,14 +792,14 @@ struct RfKernel {
         }
       }
     } else if (active) {
-      T *Bb = reinterpret_cast<T *>(p.B) + c_mat(c) * p.strideB;
+      T *Bb = reinterpret_cast<T *>(p.B) + c_mat(p, c) * p.strideB;
 #pragma unroll
       for (int i = 0; i < MR; ++i)
 #pragma unroll
         for (int j = 0; j < NC; ++j) {
           const int r = c.rg + R * i, col = c.cg + G * j;
           if (inb(r, col, m, n)) Ab[r + (long long)col * p.lda] = a[i][j];
-          if (!EX && r < m && col >= n && col < n + p.nrhs) Bb[r + (long long)(col - n) * p.ldb] = a[i][j];
+          if (AUG && r < m && col >= n && col < n + p.nrhs) Bb[r + (long long)(col - n) * p.ldb] = a[i][j];
         }
     }
   }
@@ -809,7 +821,6 @@ struct RfKernel {
     long long mat = (long long)blockIdx.x * GPB + grp;
     const bool active = mat < p.batch;
     if (!active) mat = p.batch - 1;
-    c.mat = mat;
     float *gs = smem + grp * Cfg::kSmallWords;
     c.vbuf = reinterpret_cast<T *>(gs);
     c.taus = c.vbuf + NBUF * VB;
@@ -846,15 +857,15 @@ struct RfKernel {
   }
 };
 
-template <class T, int R, int G, int MR, int NC, int GPB, bool STAGE, bool EX>
+template <class T, int R, int G, int MR, int NC, int GPB, bool STAGE, bool EX, bool AUG>
 __global__ void __launch_bounds__(R * G * GPB, 1) geqrf_rf_kernel(const RfArgs p) {
-  RfKernel<T, R, G, MR, NC, GPB, STAGE, EX>::template run<false>(p);
+  RfKernel<T, R, G, MR, NC, GPB, STAGE, EX, AUG>::template run<false>(p);
 }
 
 // p.kmax = k (reflectors), p.n = columns of Q, p.tau read-only
-template <class T, int R, int G, int MR, int NC, int GPB, bool STAGE, bool EX>
+template <class T, int R, int G, int MR, int NC, int GPB, bool STAGE, bool EX, bool AUG>
 __global__ void __launch_bounds__(R * G * GPB, 1) orgqr_rf_kernel(const RfArgs p) {
-  RfKernel<T, R, G, MR, NC, GPB, STAGE, EX>::template run<true>(p);
+  RfKernel<T, R, G, MR, NC, GPB, STAGE, EX, AUG>::template run<true>(p);
 }
 
 }  // namespace bqr
