@@ -33,18 +33,31 @@ int current_device() {
   return d < 0 ? 0 : (d >= kMaxDevices ? kMaxDevices - 1 : d);
 }
 
-// Raise a kernel's dynamic-smem limit once per (kernel, device).
-template <class K>
-bool ensure_smem(K kern, size_t smem) {
-  static std::atomic<size_t> set_bytes[kMaxDevices];
+// Raise a kernel's dynamic-smem limit once per (kernel, device).  Keyed by
+// the kernel's address: every rf instantiation has the same function type.
+bool ensure_smem(const void *kern, size_t smem) {
   if (smem <= 48 * 1024) return true;
+  struct Entry {
+    const void *k;
+    int dev;
+    size_t bytes;
+  };
+  static std::mutex mu;
+  static Entry table[512];
+  static int used = 0;
   const int d = current_device();
-  if (set_bytes[d].load(std::memory_order_acquire) >= smem) return true;
+  std::lock_guard<std::mutex> lock(mu);
+  for (int i = 0; i < used; ++i)
+    if (table[i].k == kern && table[i].dev == d) {
+      if (table[i].bytes >= smem) return true;
+      if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess)
+        return false;
+      table[i].bytes = smem;
+      return true;
+    }
   if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess)
     return false;
-  size_t cur = set_bytes[d].load();
-  while (cur < smem && !set_bytes[d].compare_exchange_weak(cur, smem)) {
-  }
+  if (used < 512) table[used++] = Entry{kern, d, smem};
   return true;
 }
 
@@ -102,10 +115,26 @@ int launch_rf(const Call &c) {
   a.strideT = c.strideT >= 0 ? c.strideT : (long long)c.k;
   a.strideB = (long long)c.ldb * c.nrhs;
   if (c.strideA >= 0) a.bulk = 0;  // panel views are not contiguous matrices
-  const size_t smem = (size_t)Cfg::kSmallAll * 4 + (STAGE ? (size_t)GPB * a.tileWords * 4 : 0);
+  // multi-warp geqrf kernels run a persistent matrix loop with a TMA-bulk
+  // prefetch of the next contiguous matrix into a shared-memory tile
+  constexpr bool kLoop = (R * G > 32) && !STAGE && !ORG;
+  const size_t mat_bytes = (size_t)c.m * c.n * sizeof(T);
+  const bool prefetch = kLoop && c.strideA == -1 && c.lda == c.m && aligned && mat_bytes % 16 == 0 &&
+                        (size_t)Cfg::kSmallAll * 4 + mat_bytes <= 200 * 1024;
+  if (kLoop) a.bulk = prefetch ? 1 : 0;
+  const size_t smem = (size_t)Cfg::kSmallAll * 4 + (STAGE ? (size_t)GPB * a.tileWords * 4 : 0) +
+                      (prefetch ? mat_bytes : 0);
   auto kern = ORG ? orgqr_rf_kernel<T, R, G, MR, NC, GPB, STAGE, EX, AUG> : geqrf_rf_kernel<T, R, G, MR, NC, GPB, STAGE, EX, AUG>;
-  if (!ensure_smem(kern, smem)) return BQR_ERR_CUDA;
-  const long long grid = (c.batch + GPB - 1) / GPB;
+  if (!ensure_smem(reinterpret_cast<const void *>(kern), smem)) return BQR_ERR_CUDA;
+  long long grid = (c.batch + GPB - 1) / GPB;
+  if (prefetch) {
+    // persistent grid: resident CTAs only (occupancy depends on smem, i.e.
+    // on the shape, so it is queried per call; host-only, no sync)
+    int sms = 0, bps = 0;
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, current_device());
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, kern, Cfg::NT, smem);
+    grid = std::min<long long>(grid, std::max(1, sms * std::max(1, bps)));
+  }
   if (grid > 0x7fffffffLL) return BQR_ERR_NOT_SUPPORTED;
   kern<<<(unsigned)grid, Cfg::NT, smem, c.stream>>>(a);
   return finish_launch();

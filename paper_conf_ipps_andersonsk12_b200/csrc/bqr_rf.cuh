@@ -377,13 +377,33 @@ struct RfKernel {
           for (int j = 0; j < NS; ++j) w[j][(i - I0) % ACC] = X::cfma(v[i], a[i][J0 + j], w[j][(i - I0) % ACC]);
       }
       T tw[NS];
+      T sum[NS];
 #pragma unroll
       for (int j = 0; j < NS; ++j) {
         T s = w[j][0];
 #pragma unroll
         for (int q = 1; q < ACC; ++q) s = X::add(s, w[j][q]);
-        s = row_allreduce<R>(s);
-        tw[j] = X::mul(ct, s);
+        sum[j] = s;
+      }
+      if constexpr (R >= 8 && NS * Cfg::E >= 2) {
+        // several values over >= 8 row lanes: reduce-scatter + all-gather
+        float f[NS * Cfg::E];
+#pragma unroll
+        for (int j = 0; j < NS; ++j)
+#pragma unroll
+          for (int e = 0; e < Cfg::E; ++e) f[j * Cfg::E + e] = get_word(sum[j], e);
+        row_allreduce_multi<R, NS * Cfg::E>(f, c.lane);
+#pragma unroll
+        for (int j = 0; j < NS; ++j)
+#pragma unroll
+          for (int e = 0; e < Cfg::E; ++e) set_word(sum[j], e, f[j * Cfg::E + e]);
+      } else {
+#pragma unroll
+        for (int j = 0; j < NS; ++j) sum[j] = row_allreduce<R>(sum[j]);
+      }
+#pragma unroll
+      for (int j = 0; j < NS; ++j) {
+        tw[j] = X::mul(ct, sum[j]);
         if (J0 + j == P) tw[j] = X::sel(c.cg > kk, tw[j], X::zero());
       }
       {
@@ -804,8 +824,85 @@ struct RfKernel {
     }
   }
 
+  // ====================================================================
+  // Persistent CTA loop (multi-warp groups, direct staging): the CTA walks
+  // matrices blockIdx.x, +gridDim.x, ...; while it factors one, a TMA bulk
+  // copy prefetches the next contiguous matrix into shared memory, so only
+  // the first load per CTA is exposed (STAP: 256 matrices on 148 SMs, the
+  // second matrix of an SM used to wait ~µs for HBM with the SM idle).
+  // ====================================================================
+  static __device__ __forceinline__ void run_cta_loop(const RfArgs &p) {
+    extern __shared__ __align__(16) float smem[];
+    const int t = threadIdx.x;
+    Ctx c;
+    c.t = t;
+    c.grp = 0;
+    c.rg = t % R;
+    c.cg = t / R;
+    c.lane = t & 31;
+    c.wid = __shfl_sync(0xffffffffu, t >> 5, 0);
+    c.kmax = p.kmax;
+    c.vbuf = reinterpret_cast<T *>(smem);
+    c.taus = c.vbuf + NBUF * VB;
+    T *tile = reinterpret_cast<T *>(smem + Cfg::kSmallAll);
+    void *bar = smem + Cfg::kMbarWord;
+    const int m = p.m, n = p.n;
+    if (p.bulk) {
+      if (t == 0) mbar_init(bar, 1);
+      __syncthreads();
+    }
+    bool have_tile = false;
+    unsigned phase = 0;
+#pragma unroll 1
+    for (long long mat = blockIdx.x; mat < p.batch; mat += gridDim.x) {
+      T *Ab = reinterpret_cast<T *>(p.A) + mat * p.strideA;
+      T a[MR][NC];
+      if (have_tile) {
+        while (!mbar_try_wait(bar, phase)) {
+        }
+        phase ^= 1;
+#pragma unroll
+        for (int i = 0; i < MR; ++i)
+#pragma unroll
+          for (int j = 0; j < NC; ++j) {
+            const int r = c.rg + R * i, col = c.cg + G * j;
+            a[i][j] = inb(r, col, m, n) ? tile[r + col * m] : X::zero();
+          }
+        if constexpr (AUG) {
+          const T *Bb = reinterpret_cast<const T *>(p.B) + mat * p.strideB;
+#pragma unroll
+          for (int i = 0; i < MR; ++i)
+#pragma unroll
+            for (int j = 0; j < NC; ++j) {
+              const int r = c.rg + R * i, col = c.cg + G * j;
+              if (r < m && col >= n && col < n + p.nrhs) a[i][j] = Bb[r + (long long)(col - n) * p.ldb];
+            }
+        }
+      } else {
+        load_matrix(p, c, smem, Ab, true, a);
+      }
+      __syncthreads();  // tile consumed by every thread
+      const long long nxt = mat + gridDim.x;
+      have_tile = p.bulk && nxt < p.batch;
+      if (have_tile && t == 0) {
+        fence_async_smem();
+        bulk_load(tile, reinterpret_cast<const T *>(p.A) + nxt * p.strideA, (unsigned)(m * n * sizeof(T)), bar);
+      }
+      panels<0>(c, a);
+      __syncthreads();  // every tau published before the tau store
+      store_matrix(p, c, smem, Ab, true, a);
+      T *tg = reinterpret_cast<T *>(p.tau) + mat * p.strideT;
+      for (int idx = t; idx < p.kmax; idx += GT) tg[idx] = c.taus[idx];
+      __syncthreads();  // vector/tau buffers reused by the next matrix
+    }
+  }
+
   template <bool ORG>
   static __device__ __forceinline__ void run(const RfArgs &p) {
+    if constexpr (GT > 32 && !STAGE && !ORG) {
+      run_cta_loop(p);
+      return;
+    }
     extern __shared__ __align__(16) float smem[];
     const int tid = threadIdx.x;
     const int grp = tid / GT;
