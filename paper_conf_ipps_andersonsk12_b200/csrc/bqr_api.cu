@@ -127,7 +127,10 @@ int launch_rf(const Call &c) {
   auto kern = ORG ? orgqr_rf_kernel<T, R, G, MR, NC, GPB, STAGE, EX, AUG> : geqrf_rf_kernel<T, R, G, MR, NC, GPB, STAGE, EX, AUG>;
   if (!ensure_smem(reinterpret_cast<const void *>(kern), smem)) return BQR_ERR_CUDA;
   long long grid = (c.batch + GPB - 1) / GPB;
-  if (prefetch) {
+  // sub-warp exact-shape kernels run a persistent prefetching warp loop when
+  // the batch is contiguous (a.bulk)
+  const bool warp_loop = (R * G <= 32) && (R * G * GPB == 32) && STAGE && EX && !ORG && a.bulk;
+  if (prefetch || warp_loop) {
     // persistent grid: resident CTAs only (occupancy depends on smem, i.e.
     // on the shape, so it is queried per call; host-only, no sync)
     int sms = 0, bps = 0;

@@ -603,17 +603,29 @@ struct RfKernel {
     usteps<0>(c, a, kmax);
   }
 
-  template <int P>
-  static __device__ __forceinline__ void panels(Ctx &c, T (&a)[MR][NC]) {
+  struct NoHook {
+    __device__ __forceinline__ void operator()() const {}
+  };
+
+  // panel recursion; `hook` runs once, before panel 1 (or at the end when
+  // there is a single panel) -- the persistent warp loop issues its deferred
+  // prefetch there, once the previous bulk store has surely read the tile
+  template <int P, class H = NoHook>
+  static __device__ __forceinline__ void panels(Ctx &c, T (&a)[MR][NC], const H &hook = H()) {
     if constexpr (P < NC) {
+      if constexpr (P == 1) hook();
       constexpr int I0 = (P * G) / R;
       const int kbeg = P * G;
-      if (kbeg >= c.kmax) return;
+      if (kbeg >= c.kmax) {
+        if constexpr (P == 0) hook();
+        return;
+      }
       const int kend = min(kbeg + G, c.kmax);
       panel_head<P, I0>(c, a, kbeg);
 #pragma unroll 1
       for (int k = kbeg; k < kend; ++k) step<P, I0>(c, a, k);
-      panels<P + 1>(c, a);
+      panels<P + 1>(c, a, hook);
+      if constexpr (P == 0 && NC == 1) hook();
     }
   }
 
@@ -897,11 +909,130 @@ struct RfKernel {
     }
   }
 
+  // ====================================================================
+  // Persistent warp loop (sub-warp groups, exact contiguous shapes): each
+  // warp walks matrix groups blockIdx.x, +gridDim.x, ...  The group's
+  // shared-memory tile always holds the NEXT input (TMA bulk prefetch, issued
+  // while the current matrix is factored); at the end of a matrix every lane
+  // swaps its result elements with the next input's elements at the same
+  // positions (so the tile becomes the output, the registers the next input),
+  // a bulk store drains the tile, and the prefetch after that is deferred to
+  // panel 1 of the next factorisation.  Loads and stores overlap compute
+  // except for the very first load and last store of a warp.
+  // ====================================================================
+  static __device__ __forceinline__ void run_warp_loop(const RfArgs &p) {
+    extern __shared__ __align__(16) float smem[];
+    const int tid = threadIdx.x;
+    const int grp = tid / GT;
+    const int t = tid - grp * GT;
+    Ctx c;
+    c.t = t;
+    c.grp = grp;
+    c.rg = t % R;
+    c.cg = t / R;
+    c.lane = tid & 31;
+    c.wid = 0;
+    c.kmax = MMAX_ < NMAX_ ? MMAX_ : NMAX_;
+    c.vbuf = reinterpret_cast<T *>(smem + grp * Cfg::kSmallWords);
+    c.taus = c.vbuf + NBUF * VB;
+    float *tile = smem + Cfg::kSmallAll + grp * p.tileWords;
+    void *bar = smem + grp * Cfg::kSmallWords + Cfg::kMbarWord;
+    constexpr int LD = MMAX_;
+    constexpr unsigned kBytes = MMAX_ * NMAX_ * 4;
+    const long long nitems = (p.batch + GPB - 1) / GPB;
+    auto matof = [&](long long q) { return q * GPB + grp; };
+    auto gptr = [&](long long mat) { return reinterpret_cast<float *>(p.A) + mat * p.strideA; };
+    if (t == 0) mbar_init(bar, 1);
+    warp_sync();
+    long long q = blockIdx.x;
+    if (q >= nitems) return;
+    // every lane waits on ALL groups' barriers of its warp: converged exit
+    auto wait_tiles = [&](unsigned phase, long long item) {
+      bool done = false;
+      while (!done) {
+        done = true;
+#pragma unroll
+        for (int g = 0; g < GPB; ++g) {
+          void *bg = smem + g * Cfg::kSmallWords + Cfg::kMbarWord;
+          if (item * GPB + g < p.batch) done = mbar_try_wait(bg, phase) && done;
+        }
+      }
+    };
+    unsigned phase = 0;
+    if (t == 0 && matof(q) < p.batch) bulk_load(tile, gptr(matof(q)), kBytes, bar);
+    wait_tiles(phase, q);
+    phase ^= 1;
+    T a[MR][NC];
+#pragma unroll
+    for (int i = 0; i < MR; ++i)
+#pragma unroll
+      for (int j = 0; j < NC; ++j) a[i][j] = tile[(c.rg + R * i) + (c.cg + G * j) * LD];
+    warp_sync();
+    long long pending = q + gridDim.x;  // prefetch target, issued at the hook
+    if (pending < nitems) {
+      if (t == 0 && matof(pending) < p.batch) bulk_load(tile, gptr(matof(pending)), kBytes, bar);
+      pending = -1;
+    }
+#pragma unroll 1
+    for (; q < nitems; q += gridDim.x) {
+      const long long mat = matof(q);
+      const bool valid = mat < p.batch;
+      auto hook = [&]() {
+        if (pending >= 0) {
+          if (t == 0) {
+            bulk_store_drain();  // the previous output left the tile
+            if (matof(pending) < p.batch) bulk_load(tile, gptr(matof(pending)), kBytes, bar);
+          }
+          pending = -1;
+        }
+      };
+      panels<0>(c, a, hook);
+      warp_sync();
+      const long long qn = q + gridDim.x;
+      if (qn < nitems) {
+        wait_tiles(phase, qn);
+        phase ^= 1;
+#pragma unroll
+        for (int i = 0; i < MR; ++i)
+#pragma unroll
+          for (int j = 0; j < NC; ++j) {
+            float *e = tile + (c.rg + R * i) + (c.cg + G * j) * LD;
+            const float x = *e;
+            *e = a[i][j];
+            a[i][j] = x;
+          }
+      } else {
+#pragma unroll
+        for (int i = 0; i < MR; ++i)
+#pragma unroll
+          for (int j = 0; j < NC; ++j) tile[(c.rg + R * i) + (c.cg + G * j) * LD] = a[i][j];
+      }
+      fence_async_smem();
+      warp_sync();
+      if (t == 0 && valid) {
+        bulk_store(gptr(mat), tile, kBytes);
+      }
+      if (valid) {
+        T *tg = reinterpret_cast<T *>(p.tau) + mat * p.strideT;
+        for (int idx = t; idx < c.kmax; idx += GT) tg[idx] = c.taus[idx];
+      }
+      warp_sync();
+      if (qn + gridDim.x < nitems) pending = qn + gridDim.x;
+    }
+    if (t == 0) bulk_store_drain();
+  }
+
   template <bool ORG>
   static __device__ __forceinline__ void run(const RfArgs &p) {
     if constexpr (GT > 32 && !STAGE && !ORG) {
       run_cta_loop(p);
       return;
+    }
+    if constexpr (GT <= 32 && GT * GPB == 32 && STAGE && EX && !ORG && Cfg::E == 1) {
+      if (p.bulk) {  // contiguous, aligned batch: persistent prefetching loop
+        run_warp_loop(p);
+        return;
+      }
     }
     extern __shared__ __align__(16) float smem[];
     const int tid = threadIdx.x;
