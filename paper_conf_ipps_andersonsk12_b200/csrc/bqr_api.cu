@@ -182,7 +182,8 @@ struct ClassEntry {
 // then the smallest class that holds (m, n).
 const ClassEntry kClasses[] = {
     // headline shapes, exact fits
-    {BQR_R32, 56, 56, 56, 56, false, RF_PLAN_X(float, 2, 8, 28, 7, 2, true, true, "rf_f32_R2G8_28x7_x2_exact")},
+    {BQR_R32, 56, 56, 56, 56, false, RF_PLAN_X(float, 4, 4, 14, 14, 2, true, true, "rf_f32_R4G4_14x14_x2_exact")},
+    {BQR_R32, 56, 56, 56, 56, true, RF_PLAN_X(float, 2, 8, 28, 7, 2, true, true, "rf_f32_R2G8_28x7_x2_exact")},
     {BQR_R32, 56, 56, 56, 56, true, RF_PLAN(float, 2, 8, 28, 7, 2, true, "rf_f32_R2G8_28x7_x2_stage")},
     {BQR_C64, 240, 66, 240, 66, false, RF_PLAN(float2, 32, 11, 8, 6, 1, false, "rf_c64_R32G11_8x6_cta")},
     {BQR_C64, 240, 66, 240, 66, true, RF_PLAN(float2, 16, 22, 15, 3, 1, false, "rf_c64_R16G22_15x3_cta")},
@@ -194,7 +195,7 @@ const ClassEntry kClasses[] = {
     {BQR_R32, 128, 128, 0, 0, true, RF_PLAN_AUG(float, 32, 8, 4, 16, "rf_f32_R32G8_4x16_aug")},
     // alternatives kept for measurement (BQR_FORCE_VARIANT)
     {BQR_R32, 56, 56, 56, 56, true, RF_PLAN(float, 4, 8, 14, 7, 1, true, "rf_f32_R4G8_14x7_x1_stage")},
-    {BQR_R32, 56, 56, 56, 56, true, RF_PLAN(float, 4, 4, 14, 14, 2, true, "rf_f32_R4G4_14x14_x2_stage")},
+
     {BQR_C64, 240, 66, 240, 66, true, RF_PLAN(float2, 32, 16, 8, 5, 1, false, "rf_c64_R32G16_8x5_cta")},
     // fp32 classes
     {BQR_R32, 16, 16, 0, 0, false, RF_PLAN(float, 2, 4, 8, 4, 8, true, "rf_f32_R2G4_8x4_x8_stage")},

@@ -359,10 +359,11 @@ struct RfKernel {
   static __device__ __forceinline__ void apply(Ctx &c, T (&a)[MR][NC], const T *vb, T ct, int kk) {
     if constexpr (J0 < J1) {
       constexpr int NS = J1 - J0;
-      // 4 partial sums per slot: ptxas walks the slots one after another, so
-      // a single accumulator per slot is a 4-cycle-per-row serial chain
-      // (measured: fewer accumulators are slower even for 8 rows per lane)
-      constexpr int ACC = 4;
+      // partial sums per slot: ptxas walks the slots one after another, so a
+      // single accumulator per slot is a 4-cycle-per-row serial chain; 4 is
+      // best when few slots are live (measured on C3/C4), fewer with many
+      // slots to bound the accumulator registers (NS x ACC)
+      constexpr int ACC = NS <= 6 ? 4 : (NS <= 12 ? 2 : 1);
       T w[NS][ACC];
 #pragma unroll
       for (int j = 0; j < NS; ++j)
