@@ -183,31 +183,32 @@ struct ClassEntry {
 const ClassEntry kClasses[] = {
     // headline shapes, exact fits
     {BQR_R32, 56, 56, 56, 56, false, RF_PLAN_X(float, 4, 4, 14, 14, 2, true, true, "rf_f32_R4G4_14x14_x2_exact")},
-    {BQR_R32, 56, 56, 56, 56, true, RF_PLAN_X(float, 2, 8, 28, 7, 2, true, true, "rf_f32_R2G8_28x7_x2_exact")},
-    {BQR_R32, 56, 56, 56, 56, true, RF_PLAN(float, 2, 8, 28, 7, 2, true, "rf_f32_R2G8_28x7_x2_stage")},
     {BQR_C64, 240, 66, 240, 66, false, RF_PLAN(float2, 32, 11, 8, 6, 1, false, "rf_c64_R32G11_8x6_cta")},
-    {BQR_C64, 240, 66, 240, 66, true, RF_PLAN(float2, 16, 22, 15, 3, 1, false, "rf_c64_R16G22_15x3_cta")},
-    {BQR_C64, 256, 72, 240, 66, true, RF_PLAN(float2, 32, 8, 8, 9, 1, false, "rf_c64_R32G8_8x9_cta")},
-    {BQR_C64, 240, 80, 240, 66, true, RF_PLAN(float2, 16, 16, 15, 5, 1, false, "rf_c64_R16G16_15x5_cta")},
-    // 240x66 with up to 6 augmented right-hand sides (fused Q^H B)
+    // augmented classes (fused Q^H B): 240x66 + up to 6 rhs, <=128 squares
     {BQR_C64, 256, 72, 240, 67, true, RF_PLAN_AUG(float2, 32, 12, 8, 6, "rf_c64_R32G12_8x6_aug")},
     {BQR_C64, 128, 128, 0, 0, true, RF_PLAN_AUG(float2, 32, 16, 4, 8, "rf_c64_R32G16_4x8_aug")},
     {BQR_R32, 128, 128, 0, 0, true, RF_PLAN_AUG(float, 32, 8, 4, 16, "rf_f32_R32G8_4x16_aug")},
     // alternatives kept for measurement (BQR_FORCE_VARIANT)
-    {BQR_R32, 56, 56, 56, 56, true, RF_PLAN(float, 4, 8, 14, 7, 1, true, "rf_f32_R4G8_14x7_x1_stage")},
-
+    {BQR_R32, 56, 56, 56, 56, true, RF_PLAN_X(float, 2, 8, 28, 7, 2, true, true, "rf_f32_R2G8_28x7_x2_exact")},
     {BQR_C64, 240, 66, 240, 66, true, RF_PLAN(float2, 32, 16, 8, 5, 1, false, "rf_c64_R32G16_8x5_cta")},
-    // fp32 classes
-    {BQR_R32, 16, 16, 0, 0, false, RF_PLAN(float, 2, 4, 8, 4, 8, true, "rf_f32_R2G4_8x4_x8_stage")},
-    {BQR_R32, 32, 32, 0, 0, false, RF_PLAN(float, 2, 8, 16, 4, 4, true, "rf_f32_R2G8_16x4_x4_stage")},
+    // fp32 classes: square R x G lane grids where the register budget allows
+    // (one pivot-mask row per panel), several matrices per warp when small
+    {BQR_R32, 16, 16, 0, 0, false, RF_PLAN(float, 2, 2, 8, 8, 8, true, "rf_f32_R2G2_8x8_x8_stage")},
+    {BQR_R32, 24, 24, 0, 0, false, RF_PLAN(float, 2, 2, 12, 12, 8, true, "rf_f32_R2G2_12x12_x8_stage")},
+    {BQR_R32, 32, 32, 0, 0, false, RF_PLAN(float, 2, 4, 16, 8, 4, true, "rf_f32_R2G4_16x8_x4_stage")},
+    {BQR_R32, 48, 48, 0, 0, false, RF_PLAN(float, 4, 4, 12, 12, 2, true, "rf_f32_R4G4_12x12_x2_stage")},
     {BQR_R32, 64, 64, 0, 0, false, RF_PLAN(float, 4, 8, 16, 8, 2, true, "rf_f32_R4G8_16x8_x2_stage")},
-    {BQR_R32, 128, 128, 0, 0, false, RF_PLAN(float, 32, 8, 4, 16, 1, false, "rf_f32_R32G8_4x16_cta")},
+    {BQR_R32, 80, 80, 0, 0, false, RF_PLAN(float, 8, 8, 10, 10, 1, false, "rf_f32_R8G8_10x10_cta")},
+    {BQR_R32, 96, 96, 0, 0, false, RF_PLAN(float, 8, 8, 12, 12, 1, false, "rf_f32_R8G8_12x12_cta")},
+    {BQR_R32, 128, 128, 0, 0, false, RF_PLAN(float, 16, 16, 8, 8, 1, false, "rf_f32_R16G16_8x8_cta")},
     {BQR_R32, 256, 64, 0, 0, false, RF_PLAN(float, 32, 8, 8, 8, 1, false, "rf_f32_R32G8_8x8_cta")},
     // complex64 classes
-    {BQR_C64, 16, 16, 0, 0, false, RF_PLAN(float2, 8, 4, 2, 4, 1, false, "rf_c64_R8G4_2x4_warp")},
-    {BQR_C64, 32, 32, 0, 0, false, RF_PLAN(float2, 8, 4, 4, 8, 1, false, "rf_c64_R8G4_4x8_warp")},
-    {BQR_C64, 64, 64, 0, 0, false, RF_PLAN(float2, 16, 8, 4, 8, 1, false, "rf_c64_R16G8_4x8_cta")},
-    {BQR_C64, 128, 128, 0, 0, false, RF_PLAN(float2, 32, 16, 4, 8, 1, false, "rf_c64_R32G16_4x8_cta")},
+    {BQR_C64, 16, 16, 0, 0, false, RF_PLAN(float2, 2, 2, 8, 8, 8, false, "rf_c64_R2G2_8x8_x8_warp")},
+    {BQR_C64, 32, 32, 0, 0, false, RF_PLAN(float2, 4, 4, 8, 8, 2, false, "rf_c64_R4G4_8x8_x2_warp")},
+    {BQR_C64, 48, 48, 0, 0, false, RF_PLAN(float2, 8, 8, 6, 6, 1, false, "rf_c64_R8G8_6x6_cta")},
+    {BQR_C64, 64, 64, 0, 0, false, RF_PLAN(float2, 8, 8, 8, 8, 1, false, "rf_c64_R8G8_8x8_cta")},
+    {BQR_C64, 96, 96, 0, 0, false, RF_PLAN(float2, 16, 16, 6, 6, 1, false, "rf_c64_R16G16_6x6_cta")},
+    {BQR_C64, 128, 128, 0, 0, false, RF_PLAN(float2, 16, 16, 8, 8, 1, false, "rf_c64_R16G16_8x8_cta")},
     {BQR_C64, 256, 96, 0, 0, false, RF_PLAN(float2, 32, 16, 8, 6, 1, false, "rf_c64_R32G16_8x6_cta")},
 };
 

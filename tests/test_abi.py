@@ -106,7 +106,7 @@ def test_status_strings(lib):
 @pytest.mark.parametrize("dt,m,n,expect", [
     (0, 4, 4, "tiny"), (0, 8, 8, "tiny"), (1, 8, 8, "tiny"),
     (0, 56, 56, "rf_f32_R4G4_14x14_x2_exact"), (1, 240, 66, "rf_c64_R32G11_8x6_cta"),
-    (0, 16, 16, "rf_f32"), (1, 100, 100, "rf_c64"),
+    (0, 16, 16, "rf_f32"), (1, 100, 100, "rf_c64"), (1, 64, 64, "rf_c64_R8G8"), (0, 80, 80, "rf_f32_R8G8"),
 ])
 def test_dispatch(lib, dt, m, n, expect):
     assert bqr.kernel_name(dt, m, n).startswith(expect)
