@@ -34,13 +34,29 @@ def stale() -> bool:
 
 
 def build(force: bool = False, verbose: bool = False, extra=()) -> str:
+    """Compile every csrc/*.cu translation unit in parallel, link libbqr.so."""
     if not force and not stale():
         return LIB
-    cmd = [NVCC, *FLAGS, *extra, "-o", LIB + ".tmp", os.path.join(CSRC, "bqr_api.cu")]
-    if verbose:
-        cmd.insert(1, "-Xptxas=-v")
-        print(" ".join(cmd), file=sys.stderr)
-    subprocess.check_call(cmd)
+    units = sorted(f for f in os.listdir(CSRC) if f.endswith(".cu"))
+    objdir = os.path.join(HERE, "build_obj")
+    os.makedirs(objdir, exist_ok=True)
+    cflags = [f for f in FLAGS if f != "-shared"]
+    procs = []
+    for u in units:
+        obj = os.path.join(objdir, u[:-3] + ".o")
+        cmd = [NVCC, *cflags, *extra, "-c", "-o", obj, os.path.join(CSRC, u)]
+        if verbose:
+            cmd.insert(1, "-Xptxas=-v")
+            print(" ".join(cmd), file=sys.stderr)
+        procs.append((u, obj, subprocess.Popen(cmd)))
+    objs = []
+    for u, obj, pr in procs:
+        if pr.wait() != 0:
+            raise subprocess.CalledProcessError(pr.returncode, f"nvcc {u}")
+        objs.append(obj)
+    link = [NVCC, "-shared", "-gencode", "arch=compute_100a,code=sm_100a", "-Xcompiler", "-fPIC",
+            "-o", LIB + ".tmp", *objs]
+    subprocess.check_call(link)
     os.replace(LIB + ".tmp", LIB)
     return LIB
 

@@ -1,0 +1,28 @@
+// bqr_classes_c64.cu -- complex64 size classes
+// (one translation unit per table so the template instantiations of the
+// size classes compile in parallel; see bqr_launch.cuh)
+#include "bqr_launch.cuh"
+
+namespace bqr {
+namespace host {
+
+namespace {
+const ClassEntry kTable[] = {
+    {BQR_C64, 16, 16, 0, 0, false, RF_PLAN(float2, 2, 2, 8, 8, 8, false, "rf_c64_R2G2_8x8_x8_warp")},
+    {BQR_C64, 32, 32, 0, 0, false, RF_PLAN(float2, 4, 4, 8, 8, 2, false, "rf_c64_R4G4_8x8_x2_warp")},
+    {BQR_C64, 48, 48, 0, 0, false, RF_PLAN(float2, 8, 8, 6, 6, 1, false, "rf_c64_R8G8_6x6_cta")},
+    {BQR_C64, 64, 64, 0, 0, false, RF_PLAN(float2, 8, 8, 8, 8, 1, false, "rf_c64_R8G8_8x8_cta")},
+    {BQR_C64, 80, 80, 0, 0, false, RF_PLAN(float2, 8, 8, 10, 10, 1, false, "rf_c64_R8G8_10x10_cta")},
+    {BQR_C64, 96, 96, 0, 0, false, RF_PLAN(float2, 16, 16, 6, 6, 1, false, "rf_c64_R16G16_6x6_cta")},
+    {BQR_C64, 128, 128, 0, 0, false, RF_PLAN(float2, 16, 16, 8, 8, 1, false, "rf_c64_R16G16_8x8_cta")},
+    {BQR_C64, 256, 96, 0, 0, false, RF_PLAN(float2, 32, 16, 8, 6, 1, false, "rf_c64_R32G16_8x6_cta")},
+};
+}  // namespace
+
+const ClassEntry *classes_c64(int *n) {
+  *n = (int)(sizeof(kTable) / sizeof(kTable[0]));
+  return kTable;
+}
+
+}  // namespace host
+}  // namespace bqr

@@ -109,3 +109,30 @@ def test_apply_and_orgqr_comparators():
     assert compare_orgqr(out, 12, 5, tau, Q.astype(np.complex64))["ok"]
     Q[0, 1, 1] += 1e-3
     assert not compare_orgqr(out, 12, 5, tau, Q)["ok"]
+
+
+def test_accepts_cascade_after_tie_flip():
+    """A factorisation that takes the other sign at a near-tie pivot (column
+    0, alpha ~ 0) legitimately differs in later pivot signs: accepted."""
+    rng = np.random.default_rng(21)
+    m = n = 8
+    A = rng.standard_normal((m, n))
+    A[0, 0] = 1e-9  # |alpha| / nu ~ 1e-9: the sign rule is a coin toss here
+    R = A.copy()
+    taus = []
+    for i in range(n):
+        alpha, x = R[i, i], R[i + 1:, i]
+        nu = np.sqrt(alpha ** 2 + x @ x)
+        beta = np.copysign(nu, alpha) if i == 0 else -np.copysign(nu, alpha)  # other sign at the tie
+        tau = (beta - alpha) / beta if x.size else 0.0
+        v = np.concatenate([[1.0], x / (alpha - beta)]) if x.size else np.array([1.0])
+        if x.size:
+            R[i + 1:, i] = v[1:]
+            R[i, i] = beta
+            C = R[i:, i + 1:]
+            C -= tau * np.outer(v, v @ C)
+        taus.append(tau)
+    A_cm = oracle.to_cm(A[None].astype(np.float32))
+    out_cm = oracle.to_cm(R[None].astype(np.float32))
+    rep = compare_geqrf(A_cm, m, out_cm, np.array([taus], dtype=np.float32))
+    assert rep["flips"] >= 1 and rep["ok"], rep

@@ -27,7 +27,10 @@ def main():
     ap.add_argument("--dtypes", default="f32,c64")
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--max-gib", type=float, default=1.0)
+    ap.add_argument("--variant", default="", help="BQR_FORCE_VARIANT for every cell")
     args = ap.parse_args()
+    if args.variant:
+        os.environ["BQR_FORCE_VARIANT"] = args.variant
     torch.cuda.set_device(0)
     props = torch.cuda.get_device_properties(0)
     n_sm = props.multi_processor_count
