@@ -58,25 +58,28 @@ using namespace bqr;
 using namespace bqr::host;
 
 // All size classes, in dispatch order: headline exact shapes and augmented
-// classes, then fp32, then complex64.
+// classes, then fp32, then complex64, then the
+// experiment-only alternatives (BQR_FORCE_VARIANT).
 struct Tables {
-  const ClassEntry *t[3];
-  int n[3];
+  static constexpr int kN = 4;
+  const ClassEntry *t[kN];
+  int n[kN];
   Tables() {
     t[0] = classes_headline(&n[0]);
     t[1] = classes_f32(&n[1]);
     t[2] = classes_c64(&n[2]);
+    t[3] = classes_alt(&n[3]);
   }
   template <class F>
   const Plan *find(F pred) const {
-    for (int a = 0; a < 3; ++a)
+    for (int a = 0; a < kN; ++a)
       for (int i = 0; i < n[a]; ++i)
         if (pred(t[a][i])) return &t[a][i].plan;
     return nullptr;
   }
   template <class F>
   void each(F f) const {
-    for (int a = 0; a < 3; ++a)
+    for (int a = 0; a < kN; ++a)
       for (int i = 0; i < n[a]; ++i) f(t[a][i]);
   }
 };

@@ -14,8 +14,11 @@ const ClassEntry kTable[] = {
     {BQR_C64, 64, 64, 0, 0, false, RF_PLAN(float2, 8, 8, 8, 8, 1, false, "rf_c64_R8G8_8x8_cta")},
     {BQR_C64, 80, 80, 0, 0, false, RF_PLAN(float2, 8, 8, 10, 10, 1, false, "rf_c64_R8G8_10x10_cta")},
     {BQR_C64, 96, 96, 0, 0, false, RF_PLAN(float2, 16, 16, 6, 6, 1, false, "rf_c64_R16G16_6x6_cta")},
+    {BQR_C64, 112, 112, 0, 0, false, RF_PLAN(float2, 16, 16, 7, 7, 1, false, "rf_c64_R16G16_7x7_cta")},
     {BQR_C64, 128, 128, 0, 0, false, RF_PLAN(float2, 16, 16, 8, 8, 1, false, "rf_c64_R16G16_8x8_cta")},
     {BQR_C64, 256, 96, 0, 0, false, RF_PLAN(float2, 32, 16, 8, 6, 1, false, "rf_c64_R32G16_8x6_cta")},
+    // 160 x 160 complex (51 K words): whole matrix in one SM's register file
+    {BQR_C64, 160, 160, 0, 0, false, RF_PLAN(float2, 16, 32, 10, 5, 1, false, "rf_c64_R16G32_10x5_cta")},
 };
 }  // namespace
 

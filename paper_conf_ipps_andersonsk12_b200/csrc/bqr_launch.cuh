@@ -172,6 +172,7 @@ int apply_dispatch(const ApplyArgs &a, cudaStream_t s) {
 const ClassEntry *classes_headline(int *n);
 const ClassEntry *classes_f32(int *n);
 const ClassEntry *classes_c64(int *n);
+const ClassEntry *classes_alt(int *n);
 Plan tiny_plan_f32(int m, int n);
 Plan tiny_plan_c64(int m, int n);
 int apply_dispatch_f32(const ApplyArgs &a, cudaStream_t s);

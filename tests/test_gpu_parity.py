@@ -68,12 +68,14 @@ F32_SHAPES = [(1, 1), (2, 2), (3, 2), (4, 4), (5, 3), (7, 7), (8, 8), (8, 1), (9
               (16, 16), (17, 17), (20, 11), (31, 31), (32, 32), (33, 33), (40, 40), (55, 55), (56, 56),
               (57, 57), (56, 20), (63, 63), (64, 64), (65, 65), (80, 80), (96, 96), (100, 37), (127, 127),
               (128, 128), (200, 50), (256, 64),
-              # oversize: tiled panels
-              (129, 129), (160, 160), (192, 192), (224, 224), (256, 256), (256, 200), (200, 150)]
+              # 129..256: one matrix per SM, 256-1024 threads (R16G16 / R32G32 classes)
+              (129, 129), (144, 144), (140, 130), (160, 160), (161, 161), (176, 176), (192, 192), (208, 100),
+              (224, 224), (240, 240), (256, 256), (256, 200), (200, 150)]
 C64_SHAPES = [(1, 1), (2, 2), (4, 4), (5, 5), (8, 8), (8, 3), (9, 9), (16, 16), (17, 17), (32, 32), (33, 20),
               (48, 48), (64, 64), (65, 65), (80, 16), (96, 96), (128, 128), (192, 96), (240, 66), (256, 96),
-              # oversize: tiled panels
-              (160, 160), (192, 192), (224, 224), (256, 256), (129, 100)]
+              (129, 100), (150, 150), (160, 120), (160, 160),
+              # oversize (> 160 complex): tiled panels
+              (161, 161), (176, 176), (192, 192), (224, 224), (256, 256)]
 
 
 @pytest.mark.parametrize("m,n", F32_SHAPES)
@@ -88,9 +90,10 @@ def test_sweep_c64(m, n):
     _check(A, m, full_q=m <= 128)
 
 
-@pytest.mark.parametrize("dt,n", [("f32", 256), ("c64", 256), ("c64", 192)])
+@pytest.mark.parametrize("dt,n", [("f32", 256), ("f32", 160), ("c64", 160), ("c64", 256), ("c64", 192)])
 def test_oversize_lda_and_determinism(dt, n):
-    """Tiled panel views keep lda > m padding untouched and are deterministic."""
+    """Large classes and tiled panel views keep lda > m padding untouched and
+    are deterministic."""
     A = bqr_inputs.random_batch(n, n, 9, dt, seed=5, lda=n + 5)
     o1, t1 = geqrf_gpu(A, n)
     rep = compare_geqrf(A, n, o1, t1, full_q=False)
@@ -172,7 +175,8 @@ def test_non_default_stream():
 # ------------------------------------------------------------- orgqr / apply
 
 @pytest.mark.parametrize("dt,m,n", [("f32", 8, 8), ("f32", 56, 56), ("f32", 30, 12), ("f32", 128, 128),
-                                    ("c64", 16, 16), ("c64", 240, 66), ("c64", 64, 40)])
+                                    ("f32", 160, 160), ("f32", 256, 256), ("f32", 200, 120),
+                                    ("c64", 16, 16), ("c64", 240, 66), ("c64", 64, 40), ("c64", 160, 160)])
 def test_orgqr(dt, m, n):
     A = bqr_inputs.random_batch(m, n, 64, dt, seed=61)
     out, tau = geqrf_gpu(A, m)
