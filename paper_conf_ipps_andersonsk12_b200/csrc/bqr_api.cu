@@ -114,6 +114,13 @@ const Plan *pick(bqr_dtype_t dt, int m, int n) {
 // fused geqrf + Q^H B: smallest augmented class whose tile holds n + nrhs
 // columns (the augmented matrix of P:L313)
 const Plan *pick_fused(bqr_dtype_t dt, int m, int n, int nrhs) {
+  if (const char *f = forced_variant()) {
+    if (const Plan *p = tables().find([&](const ClassEntry &e) {
+          return e.dt == dt && std::strcmp(e.plan.name, f) == 0 && std::strstr(f, "_aug") && m <= e.mmax &&
+                 n + nrhs <= e.nmax;
+        }))
+      return p;
+  }
   const Plan *best = nullptr;
   int best_area = 1 << 30;
   tables().each([&](const ClassEntry &e) {
@@ -199,6 +206,8 @@ size_t elem_size(bqr_dtype_t d) { return d == BQR_R32 ? 4 : 8; }
 extern "C" {
 
 const char *bqr_version(void) { return "bqr 0.1.0 (sm_100a)"; }
+
+
 
 const char *bqr_status_string(int status) {
   if (status < 0) return "illegal argument (-i = position of the first bad argument)";

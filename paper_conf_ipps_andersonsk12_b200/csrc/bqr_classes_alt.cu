@@ -18,6 +18,17 @@ const ClassEntry kTable[] = {
     {BQR_C64, 160, 160, 0, 0, true, RF_PLAN(float2, 32, 16, 5, 10, 1, false, "alt_c64_R32G16_5x10_cta")},
     {BQR_R32, 128, 128, 0, 0, true, RF_PLAN(float, 8, 8, 16, 16, 1, false, "alt_f32_R8G8_16x16_cta")},
     {BQR_C64, 144, 144, 0, 0, true, RF_PLAN(float2, 16, 16, 9, 9, 1, false, "alt_c64_R16G16_9x9_cta")},
+    // STAP 240x66 c64: 16 row lanes (4-level butterflies) instead of 32
+    {BQR_C64, 240, 66, 240, 66, true, RF_PLAN(float2, 16, 22, 15, 3, 1, false, "alt_c64_R16G22_15x3_cta")},
+    {BQR_C64, 240, 72, 0, 0, true, RF_PLAN_AUG(float2, 16, 24, 15, 3, "alt_c64_R16G24_15x3_aug")},
+    {BQR_C64, 240, 72, 0, 0, true, RF_PLAN_AUG(float2, 16, 12, 15, 6, "alt_c64_R16G12_15x6_aug")},
+    {BQR_C64, 256, 72, 0, 0, true, RF_PLAN_AUG(float2, 32, 24, 8, 3, "alt_c64_R32G24_8x3_aug")},
+    // 56x56 fp32, one matrix per warp, register cap for MB warps per SM
+    {BQR_R32, 56, 56, 56, 56, true, RF_PLAN_XM(float, 4, 8, 14, 7, 1, true, true, 12, "alt_f32_R4G8_14x7_x1_mb12")},
+    {BQR_R32, 56, 56, 56, 56, true, RF_PLAN_XM(float, 4, 8, 14, 7, 1, true, true, 14, "alt_f32_R4G8_14x7_x1_mb14")},
+    {BQR_R32, 56, 56, 56, 56, true, RF_PLAN_XM(float, 4, 8, 14, 7, 1, true, true, 16, "alt_f32_R4G8_14x7_x1_mb16")},
+    {BQR_R32, 56, 56, 56, 56, true, RF_PLAN_XM(float, 8, 4, 7, 14, 1, true, true, 12, "alt_f32_R8G4_7x14_x1_mb12")},
+    {BQR_R32, 56, 56, 56, 56, true, RF_PLAN_XM(float, 8, 4, 7, 14, 1, true, true, 14, "alt_f32_R8G4_7x14_x1_mb14")},
 };
 }  // namespace
 

@@ -23,3 +23,15 @@ const ClassEntry *classes_headline(int *n) {
 
 }  // namespace host
 }  // namespace bqr
+
+#ifdef BQR_PHASE_TIMING
+// debug builds only: the phase-timing stamps of this translation unit's
+// kernels (the headline classes; tools/phase_timing.py)
+extern "C" int bqr_debug_stamps(void *host, size_t bytes) {
+  return cudaMemcpyFromSymbol(host, bqr::g_bqr_dbg, bytes) == cudaSuccess ? 0 : 2;
+}
+extern "C" int bqr_debug_clear(void) {
+  static unsigned long long z[bqr::kDbgSteps * bqr::kDbgWarps * 4];
+  return cudaMemcpyToSymbol(bqr::g_bqr_dbg, z, sizeof(z)) == cudaSuccess ? 0 : 2;
+}
+#endif

@@ -56,7 +56,7 @@ inline int staging_ld(int m) {
   return (m + 3) & ~3;
 }
 
-template <class T, int R, int G, int MR, int NC, int GPB, bool STAGE, bool EX, bool AUG, bool ORG>
+template <class T, int R, int G, int MR, int NC, int GPB, bool STAGE, bool EX, bool AUG, bool ORG, int MB = 1>
 int launch_rf(const Call &c) {
   using Cfg = RfCfg<T, R, G, MR, NC, GPB, STAGE, EX>;
   if (EX && (c.m != R * MR || c.n != G * NC)) return BQR_ERR_NOT_SUPPORTED;
@@ -90,7 +90,7 @@ int launch_rf(const Call &c) {
   if (kLoop) a.bulk = prefetch ? 1 : 0;
   const size_t smem = (size_t)Cfg::kSmallAll * 4 + (STAGE ? (size_t)GPB * a.tileWords * 4 : 0) +
                       (prefetch ? mat_bytes : 0);
-  auto kern = ORG ? orgqr_rf_kernel<T, R, G, MR, NC, GPB, STAGE, EX, AUG> : geqrf_rf_kernel<T, R, G, MR, NC, GPB, STAGE, EX, AUG>;
+  auto kern = ORG ? orgqr_rf_kernel<T, R, G, MR, NC, GPB, STAGE, EX, AUG, MB> : geqrf_rf_kernel<T, R, G, MR, NC, GPB, STAGE, EX, AUG, MB>;
   if (!ensure_smem(reinterpret_cast<const void *>(kern), smem)) return BQR_ERR_CUDA;
   long long grid = (c.batch + GPB - 1) / GPB;
   // sub-warp exact-shape kernels run a persistent prefetching warp loop when
@@ -130,6 +130,12 @@ int launch_tiny(const Call &c) {
   Plan {                                                                 \
     NAME, &launch_rf<T, R, G, MR, NC, GPB, STAGE, EX, AUG, false>,       \
         &launch_rf<T, R, G, MR, NC, GPB, STAGE, EX, false, true>         \
+  }
+// MB > 1: register cap for MB resident CTAs per SM (launch bounds)
+#define RF_PLAN_XM(T, R, G, MR, NC, GPB, STAGE, EX, MB, NAME)                  \
+  Plan {                                                                     \
+    NAME, &launch_rf<T, R, G, MR, NC, GPB, STAGE, EX, false, false, MB>,     \
+        &launch_rf<T, R, G, MR, NC, GPB, STAGE, EX, false, true, MB>         \
   }
 #define RF_PLAN_X(T, R, G, MR, NC, GPB, STAGE, EX, NAME) RF_PLAN_XA(T, R, G, MR, NC, GPB, STAGE, EX, false, NAME)
 #define RF_PLAN(T, R, G, MR, NC, GPB, STAGE, NAME) RF_PLAN_X(T, R, G, MR, NC, GPB, STAGE, false, NAME)

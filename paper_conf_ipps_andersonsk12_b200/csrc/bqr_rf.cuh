@@ -33,7 +33,25 @@
 #pragma once
 #include "bqr_common.cuh"
 
+
 namespace bqr {
+
+#ifdef BQR_PHASE_TIMING
+// Debug build only (-DBQR_PHASE_TIMING): clock64 stamps of the first matrix
+// of CTA 0, [step][warp][phase]: 0 step entry, 1 after the step wait,
+// 2 after the look-ahead reflector (owner) / slot P, 3 step end.
+constexpr int kDbgSteps = 300, kDbgWarps = 32;
+static __device__ unsigned long long g_bqr_dbg[kDbgSteps * kDbgWarps * 4];  // per TU
+#define BQR_STAMP(c, k, ph)                                                                \
+  do {                                                                                     \
+    if ((c).dbg && ((c).lane == 0) && (k) < kDbgSteps)                                     \
+      g_bqr_dbg[(((k) * kDbgWarps) + ((c).t >> 5)) * 4 + (ph)] = clock64();                 \
+  } while (0)
+#else
+#define BQR_STAMP(c, k, ph) \
+  do {                      \
+  } while (0)
+#endif
 
 struct RfArgs {
   void *A;
@@ -210,7 +228,11 @@ struct RfKernel {
     int rg, cg, t, lane, grp;
     int wid;   // warp index in the group, warp-uniform by construction (shfl)
     int kmax;
+#ifdef BQR_PHASE_TIMING
+    bool dbg;
+#endif
   };
+
 
   struct Look {
     T scal, tau;
@@ -435,7 +457,9 @@ struct RfKernel {
   template <int P, int I0>
   static __device__ __forceinline__ void step(Ctx &c, T (&a)[MR][NC], int k) {
     const int kk = k - P * G;
+    BQR_STAMP(c, k, 0);
     if (!warp_has(c, k) || GT <= 32) step_wait<GT, NBUF>(k);
+    BQR_STAMP(c, k, 1);
     const T ct = X::conj(c.taus[k]);
     const T *vb = c.vbuf + buf(k) * VB + c.rg * MRP;
     if (!warp_done_slot(c, kk)) apply<P, I0, P, P + 1>(c, a, vb, ct, kk);
@@ -447,6 +471,7 @@ struct RfKernel {
       const Look l = reflector<P, I0>(c, a, k + 1);
       apply<P, I0, P + 1, NC>(c, a, vb, ct, kk);
       publish<P, I0>(c, a, k + 1, l, la);
+      BQR_STAMP(c, k, 3);
     } else {
       // multi-warp groups: publish first so the other warps never wait
       if (la) {
@@ -454,7 +479,9 @@ struct RfKernel {
         publish<P, I0>(c, a, k + 1, l, true);
         step_arrive<GT, NBUF>(k + 1);
       }
+      BQR_STAMP(c, k, 2);
       apply<P, I0, P + 1, NC>(c, a, vb, ct, kk);
+      BQR_STAMP(c, k, 3);
     }
   }
 
@@ -855,6 +882,9 @@ struct RfKernel {
     c.lane = t & 31;
     c.wid = __shfl_sync(0xffffffffu, t >> 5, 0);
     c.kmax = p.kmax;
+#ifdef BQR_PHASE_TIMING
+    c.dbg = blockIdx.x == 0;
+#endif
     c.vbuf = reinterpret_cast<T *>(smem);
     c.taus = c.vbuf + NBUF * VB;
     T *tile = reinterpret_cast<T *>(smem + Cfg::kSmallAll);
@@ -902,6 +932,9 @@ struct RfKernel {
         bulk_load(tile, reinterpret_cast<const T *>(p.A) + nxt * p.strideA, (unsigned)(m * n * sizeof(T)), bar);
       }
       panels<0>(c, a);
+#ifdef BQR_PHASE_TIMING
+      c.dbg = false;
+#endif
       __syncthreads();  // every tau published before the tau store
       store_matrix(p, c, smem, Ab, true, a);
       T *tg = reinterpret_cast<T *>(p.tau) + mat * p.strideT;
@@ -934,6 +967,9 @@ struct RfKernel {
     c.lane = tid & 31;
     c.wid = 0;
     c.kmax = MMAX_ < NMAX_ ? MMAX_ : NMAX_;
+#ifdef BQR_PHASE_TIMING
+    c.dbg = blockIdx.x == 0;
+#endif
     c.vbuf = reinterpret_cast<T *>(smem + grp * Cfg::kSmallWords);
     c.taus = c.vbuf + NBUF * VB;
     float *tile = smem + Cfg::kSmallAll + grp * p.tileWords;
@@ -988,6 +1024,9 @@ struct RfKernel {
         }
       };
       panels<0>(c, a, hook);
+#ifdef BQR_PHASE_TIMING
+      c.dbg = false;
+#endif
       warp_sync();
       const long long qn = q + gridDim.x;
       if (qn < nitems) {
@@ -1086,14 +1125,16 @@ struct RfKernel {
   }
 };
 
-template <class T, int R, int G, int MR, int NC, int GPB, bool STAGE, bool EX, bool AUG>
-__global__ void __launch_bounds__(R * G * GPB, 1) geqrf_rf_kernel(const RfArgs p) {
+// MB = minimum resident CTAs per SM (launch bounds): caps the registers per
+// thread so that MB groups of a small-matrix class share an SM
+template <class T, int R, int G, int MR, int NC, int GPB, bool STAGE, bool EX, bool AUG, int MB = 1>
+__global__ void __launch_bounds__(R * G * GPB, MB) geqrf_rf_kernel(const RfArgs p) {
   RfKernel<T, R, G, MR, NC, GPB, STAGE, EX, AUG>::template run<false>(p);
 }
 
 // p.kmax = k (reflectors), p.n = columns of Q, p.tau read-only
-template <class T, int R, int G, int MR, int NC, int GPB, bool STAGE, bool EX, bool AUG>
-__global__ void __launch_bounds__(R * G * GPB, 1) orgqr_rf_kernel(const RfArgs p) {
+template <class T, int R, int G, int MR, int NC, int GPB, bool STAGE, bool EX, bool AUG, int MB = 1>
+__global__ void __launch_bounds__(R * G * GPB, MB) orgqr_rf_kernel(const RfArgs p) {
   RfKernel<T, R, G, MR, NC, GPB, STAGE, EX, AUG>::template run<true>(p);
 }
 

@@ -15,7 +15,7 @@ for nm in names:
     env = dict(os.environ, BQR_FORCE_VARIANT=nm)
     code = f"""
 import sys, json; sys.path.insert(0, {ROOT!r}); sys.path.insert(0, {os.path.join(ROOT, 'tests')!r})
-import torch, bench, numpy as np
+import os, torch, bench, numpy as np
 import paper_conf_ipps_andersonsk12_b200 as bqr
 import bqr_inputs
 from oracle.compare import compare_geqrf
@@ -28,7 +28,7 @@ w = bench.Workload({cfg!r}, 0, 1, torch, bqr)
 flush = torch.empty(256 << 20, dtype=torch.uint8, device='cuda')
 class A_: pass
 smp = bench.ClockSampler(0, 0.005)
-s_ms, q_ms = bench.time_workload(w, 50, 5, torch, None, 1, flush, sampler=smp, fused=False)
+s_ms, q_ms = bench.time_workload(w, 50, 5, torch, None, 1, flush, sampler=smp, fused=bool(int(os.environ.get('FUSED', '0'))))
 clk = smp.summary()
 print(json.dumps({{'variant': {nm!r}, 'kernel': bqr.kernel_name(w.code, w.m, w.n), 'qr_us': round(q_ms*1e3, 2),
    'step_us': round(s_ms*1e3, 2), 'gflops': round(w.flops/(q_ms/1e3)/1e9, 1), 'parity_ok': rep['ok'],
