@@ -61,6 +61,9 @@ def _load():
             for name in ("bqr_ref_apply_qh_d", "bqr_ref_apply_qh_z"):
                 getattr(lib, name).argtypes = [i, i, i, i, i64, p, i, p, p, i]
                 getattr(lib, name).restype = None
+            for name in ("bqr_ref_gels_d", "bqr_ref_gels_z"):
+                getattr(lib, name).argtypes = [i, i, i, i64, p, i, p, p, i, p]
+                getattr(lib, name).restype = None
             lib.bqr_ref_set_threads.argtypes = [i]
             lib.bqr_ref_max_threads.restype = i
             _lib = lib
@@ -180,3 +183,36 @@ def apply_qh(RV: np.ndarray, tau: np.ndarray, B: np.ndarray):
 def triu_r(RV: np.ndarray) -> np.ndarray:
     """R = upper trapezoid of the geqrf output."""
     return np.triu(RV)
+
+
+def gels_cm(A_cm: np.ndarray, m: int, B_cm: np.ndarray):
+    """Least squares min ||A x - b|| by QR (paper Sec. III-D) on
+    column-major storage: A (batch, n, lda), B (batch, nrhs, ldb), m >= n.
+    Returns (A_out_cm [R; V], tau (batch, n), B_out_cm [X; residual
+    components], info (batch,) int32: 0 or j+1 for the first zero R_jj)."""
+    lib = _load()
+    A = _widen(A_cm).copy()
+    batch, n, lda = A.shape
+    assert m >= n
+    B = np.ascontiguousarray(B_cm, dtype=A.dtype).copy()
+    _, nrhs, ldb = B.shape
+    tau = np.zeros((batch, n), dtype=A.dtype)
+    info = np.zeros((batch,), dtype=np.int32)
+    if batch and n:
+        fn = lib.bqr_ref_gels_z if _is_complex(A) else lib.bqr_ref_gels_d
+        fn(m, n, nrhs, batch, _ptr(A), lda, _ptr(tau), _ptr(B), ldb, _ptr(info))
+    return A, tau, B, info
+
+
+def gels(A: np.ndarray, B: np.ndarray):
+    """Logical API: A (batch, m, n), B (batch, m, nrhs) -> (X (batch, n, nrhs),
+    residual components (batch, m-n, nrhs), info)."""
+    A = np.asarray(A)
+    B = np.asarray(B)
+    if A.ndim == 2:
+        A, B = A[None], B[None]
+    m, n = A.shape[1], A.shape[2]
+    _, _, Bo, info = gels_cm(to_cm(A), m, to_cm(B))
+    Bl = from_cm(Bo, m)
+    return Bl[:, :n, :], Bl[:, n:, :], info
+

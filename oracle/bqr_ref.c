@@ -290,3 +290,76 @@ void bqr_ref_apply_qh_z(int m, int n, int k, int nrhs, int64_t batch,
     apply_qh_z(m, k, nrhs, Az + b * (int64_t)lda * n, lda, tz + b * k,
                Bz + b * (int64_t)ldb * nrhs, ldb);
 }
+
+/* ------------------------------------------------------------------------ */
+/* Least squares (paper Sec. III-D):                             */
+/*   "find the QR factorization of A, apply Q^T to b, and solve the          */
+/*    resulting upper triangular system for x ... We compute Q^T b by        */
+/*    appending b to the right side of the matrix during the factorization.  */
+/*    We then solve the upper triangular system using row operations."       */
+/* Here: geqr2 of A, Q^H B (the appended columns, xORM2R), then backward     */
+/* elimination on [R | c] by row operations: for j = n-1 .. 0,               */
+/* x_j = c_j / R_jj, then row j times x_j is subtracted from rows 0..j-1.    */
+/* On exit B[0:n] = X and B[n:m] = the residual components (Q^H B)[n:m]      */
+/* (LAPACK xGELS convention: ||A x - b||^2 = sum of their squares).          */
+/* info = 0, or j+1 for the first j with R_jj == 0 (solution undefined).     */
+/* ------------------------------------------------------------------------ */
+
+static int backsolve_d(int n, int nrhs, const double *R, int lda, double *B,
+                       int ldb) {
+  int info = 0;
+  for (int j = 0; j < n; ++j)
+    if (R[(size_t)j * lda + j] == 0.0 && !info) info = j + 1;
+  for (int r = 0; r < nrhs; ++r) {
+    double *c = B + (size_t)r * ldb;
+    for (int j = n - 1; j >= 0; --j) {
+      const double xj = c[j] / R[(size_t)j * lda + j];
+      c[j] = xj;
+      for (int i = 0; i < j; ++i) c[i] -= R[(size_t)j * lda + i] * xj;
+    }
+  }
+  return info;
+}
+
+static int backsolve_z(int n, int nrhs, const zc *R, int lda, zc *B, int ldb) {
+  int info = 0;
+  for (int j = 0; j < n; ++j)
+    if (R[(size_t)j * lda + j] == 0.0 && !info) info = j + 1;
+  for (int r = 0; r < nrhs; ++r) {
+    zc *c = B + (size_t)r * ldb;
+    for (int j = n - 1; j >= 0; --j) {
+      const zc xj = c[j] / R[(size_t)j * lda + j];
+      c[j] = xj;
+      for (int i = 0; i < j; ++i) c[i] -= R[(size_t)j * lda + i] * xj;
+    }
+  }
+  return info;
+}
+
+/* A (m x n, m >= n) is overwritten by its QR factorization, tau (stride n),
+ * B (m x nrhs, stride ldb*nrhs) by [X; residual components]. */
+void bqr_ref_gels_d(int m, int n, int nrhs, int64_t batch, double *A, int lda,
+                    double *tau, double *B, int ldb, int *info) {
+  OMP_FOR
+  for (int64_t b = 0; b < batch; ++b) {
+    double *Ab = A + b * (int64_t)lda * n, *Bb = B + b * (int64_t)ldb * nrhs;
+    geqr2_d(m, n, Ab, lda, tau + b * n, NULL);
+    apply_qt_d(m, n, nrhs, Ab, lda, tau + b * n, Bb, ldb);
+    const int inf = backsolve_d(n, nrhs, Ab, lda, Bb, ldb);
+    if (info) info[b] = inf;
+  }
+}
+
+void bqr_ref_gels_z(int m, int n, int nrhs, int64_t batch, double *A, int lda,
+                    double *tau, double *B, int ldb, int *info) {
+  zc *Az = (zc *)A, *tz = (zc *)tau, *Bz = (zc *)B;
+  OMP_FOR
+  for (int64_t b = 0; b < batch; ++b) {
+    zc *Ab = Az + b * (int64_t)lda * n, *Bb = Bz + b * (int64_t)ldb * nrhs;
+    geqr2_z(m, n, Ab, lda, tz + b * n, NULL);
+    apply_qh_z(m, n, nrhs, Ab, lda, tz + b * n, Bb, ldb);
+    const int inf = backsolve_z(n, nrhs, Ab, lda, Bb, ldb);
+    if (info) info[b] = inf;
+  }
+}
+
