@@ -20,12 +20,23 @@ north-star tolerances):
   5. invariants   complex diag(R) imag == 0 exactly; real tau in {0} U [1,2];
                   complex |1 - tau| <= 1.
 Tolerances are the north-star's (BASELINE.json), fixed here and in DESIGN.md.
+
+compare_gels judges the least-squares solve by
+  * info equal to the oracle's (first zero R_jj);
+  * normwise backward error of the normal equations
+        ||A^H (A x - b)||_2 / (||A||_F (||A||_F ||x||_2 + ||b||_2)) <= 1e-6
+    (fp32 LAPACK sgels/cgels reach <= 4e-8 on the parity shapes: DESIGN.md);
+  * forward error against the oracle's fp64 solution, scaled by the LS
+    condition bound kappa (1 + kappa ||r|| / (||A||_2 ||x||)), kappa =
+    cond(R_ref): <= 1e-5 (LAPACK fp32: <= 5.4e-8);
+  * the residual components: their norm equals ||A x_ref - b|| within 1e-4
+    relative (+1e-6 ||b|| absolute).
 """
 from __future__ import annotations
 
 import numpy as np
 
-from . import geqrf_cm, orgqr_cm
+from . import gels_cm, geqrf_cm, orgqr_cm
 
 RESID_TOL = 1e-5
 ORTH_TOL = 1e-5
@@ -178,3 +189,48 @@ def compare_apply(RV_cm: np.ndarray, m: int, k: int, tau: np.ndarray, B_cm: np.n
     err = diff / np.where(scale == 0, 1.0, scale)
     e = float(err.max()) if err.size else 0.0
     return {"apply_err_max": e, "ok": e <= 1e-5}
+
+
+GELS_BACKWARD_TOL = 1e-6
+GELS_FORWARD_TOL = 1e-5
+GELS_RESID_TOL = 1e-4
+
+
+def compare_gels(A_cm: np.ndarray, m: int, B_cm: np.ndarray, B_out_cm: np.ndarray, info_gpu: np.ndarray) -> dict:
+    """A_cm (batch, n, lda), B_cm (batch, nrhs, ldb) inputs; B_out_cm the GPU's
+    [X; residual components]; info_gpu (batch,)."""
+    batch, n, _ = A_cm.shape
+    Ao, _, Bo, info = gels_cm(A_cm, m, B_cm)
+    A = _logical(A_cm, m).astype(np.complex128 if np.iscomplexobj(A_cm) else np.float64)
+    B = _logical(B_cm, m).astype(A.dtype)
+    Bg = _logical(B_out_cm, m).astype(A.dtype)
+    Br = _logical(Bo, m)
+    rep = {"ok": True, "info_mismatch": int((np.asarray(info_gpu) != info).sum()), "backward_max": 0.0,
+           "forward_scaled_max": 0.0, "resid_err_max": 0.0, "n_rank_deficient": int((info != 0).sum())}
+    if rep["info_mismatch"]:
+        rep["ok"] = False
+    for b in range(batch):
+        if info[b] != 0:
+            continue
+        Ab, bb, xg, xr = A[b], B[b], Bg[b, :n], Br[b, :n]
+        nA = np.linalg.norm(Ab)
+        r = Ab @ xg - bb
+        be = np.linalg.norm(Ab.conj().T @ r) / (nA * (nA * np.linalg.norm(xg) + np.linalg.norm(bb)) + 1e-300)
+        R = np.triu(_logical(Ao, m)[b, :n, :n])
+        kap = np.linalg.cond(R)
+        rr = np.linalg.norm(Ab @ xr - bb)
+        nx = np.linalg.norm(xr)
+        bound = kap * (1 + kap * rr / (np.linalg.norm(Ab, 2) * nx + 1e-300))
+        fw = np.linalg.norm(xg - xr) / (nx + 1e-300) / bound if nx > 0 else np.linalg.norm(xg)
+        res_g = np.linalg.norm(Bg[b, n:], axis=0)
+        res_r = np.linalg.norm(Ab @ xr - bb, axis=0)
+        re = float(np.max(np.abs(res_g - res_r) / (res_r + 1e-6 * np.linalg.norm(bb) / GELS_RESID_TOL + 1e-300))) \
+            if m > n else 0.0
+        rep["backward_max"] = max(rep["backward_max"], float(be))
+        rep["forward_scaled_max"] = max(rep["forward_scaled_max"], float(fw))
+        rep["resid_err_max"] = max(rep["resid_err_max"], re)
+    if rep["backward_max"] > GELS_BACKWARD_TOL or rep["forward_scaled_max"] > GELS_FORWARD_TOL or \
+            rep["resid_err_max"] > GELS_RESID_TOL:
+        rep["ok"] = False
+    return rep
+

@@ -23,7 +23,7 @@ import os
 __all__ = [
     "load", "colmajor", "geqrf_batched", "orgqr_batched", "apply_qh_batched",
     "geqrf_batched_host", "host_workspace_bytes", "kernel_name", "geqrf_launches",
-    "BQRError", "R32", "C64", "lib_path", "geqrf_batched_ptr", "geqrf_qhb_batched",
+    "BQRError", "R32", "C64", "lib_path", "geqrf_batched_ptr", "geqrf_qhb_batched", "gels_batched",
 ]
 
 R32, C64 = 0, 1
@@ -59,6 +59,9 @@ def load():
         lib.bqr_geqrf_qhb_batched.restype = i
         lib.bqr_qhb_kernel_name.argtypes = [i, i, i, i]
         lib.bqr_qhb_kernel_name.restype = ctypes.c_char_p
+    if hasattr(lib, "bqr_gels_batched"):  # absent in older builds (A/B timing)
+        lib.bqr_gels_batched.argtypes = [i, i, i, i, i, p, i, p, p, i, p, p]
+        lib.bqr_gels_batched.restype = i
     lib.bqr_geqrf_batched_host.argtypes = [i, i, i, i, p, i, p, p, sz, p]
     lib.bqr_host_workspace_bytes.argtypes = [i, i, i, i, i]
     lib.bqr_host_workspace_bytes.restype = sz
@@ -184,6 +187,26 @@ def geqrf_qhb_batched(A, B, tau=None, stream=None):
                                       _stream_ptr(stream))
     _check(st, "bqr_geqrf_qhb_batched")
     return A, tau, B
+
+
+def gels_batched(A, B, tau=None, info=None, stream=None):
+    """Least squares by QR: A (batch, m, n) <- [R; V],
+    B (batch, m, nrhs) <- [X; residual components].  Returns (A, tau, B, info)
+    with info (batch,) int32 on the device (0, or j+1 for a zero R_jj)."""
+    import torch
+    batch, m, n = A.shape
+    m, n, lda = _layout(A)
+    _, mb, nrhs = B.shape
+    _, _, ldb = _layout(B)
+    if tau is None:
+        tau = torch.empty((batch, n), dtype=A.dtype, device=A.device)
+    if info is None:
+        info = torch.empty((batch,), dtype=torch.int32, device=A.device)
+    st = load().bqr_gels_batched(_dtype_code(A), m, n, nrhs, batch, ctypes.c_void_p(A.data_ptr()), lda,
+                                 ctypes.c_void_p(tau.data_ptr()), ctypes.c_void_p(B.data_ptr()), ldb,
+                                 ctypes.c_void_p(info.data_ptr()), _stream_ptr(stream))
+    _check(st, "bqr_gels_batched")
+    return A, tau, B, info
 
 
 def host_workspace_bytes(dtype: int, m: int, n: int, lda: int, chunk: int) -> int:

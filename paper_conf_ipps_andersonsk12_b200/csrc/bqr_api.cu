@@ -125,6 +125,7 @@ const Plan *pick_fused(bqr_dtype_t dt, int m, int n, int nrhs) {
   int best_area = 1 << 30;
   tables().each([&](const ClassEntry &e) {
     if (e.dt != dt || m > e.mmax || n + nrhs > e.nmax) return;
+    if (std::strncmp(e.plan.name, "alt_", 4) == 0) return;  // experiment-only variants (BQR_FORCE_VARIANT)
     if (!std::strstr(e.plan.name, "_aug")) return;
     const int area = e.mmax * e.nmax;
     if (area < best_area) {
@@ -304,6 +305,33 @@ int bqr_geqrf_qhb_batched(bqr_dtype_t dtype, int m, int n, int nrhs, int batch, 
   int st = bqr_geqrf_batched(dtype, m, n, batch, A, lda, tau, stream);
   if (st != BQR_SUCCESS || nrhs == 0) return st;
   return bqr_apply_qh_batched(dtype, m, n, k, nrhs, batch, A, lda, tau, B, ldb, stream);
+}
+
+int bqr_gels_batched(bqr_dtype_t dtype, int m, int n, int nrhs, int batch, void *A, int lda, void *tau, void *B,
+                     int ldb, int *info, cudaStream_t stream) {
+  if (!valid_dtype(dtype)) return -1;
+  if (m < 0) return -2;
+  if (n < 0) return -3;
+  if (nrhs < 0) return -4;
+  if (batch < 0) return -5;
+  const bool work = m > 0 && n > 0 && batch > 0;
+  if (work && A == nullptr) return -6;
+  if (lda < std::max(1, m)) return -7;
+  if (work && tau == nullptr) return -8;
+  if (work && nrhs > 0 && B == nullptr) return -9;
+  if (ldb < std::max(1, m)) return -10;
+  if (!work) return BQR_SUCCESS;
+  if (m < n) return BQR_ERR_NOT_SUPPORTED;  // minimum-norm (underdetermined) problems are not built
+  if (n > 256) return BQR_ERR_NOT_SUPPORTED;
+  if ((reinterpret_cast<uintptr_t>(A) | reinterpret_cast<uintptr_t>(tau) | reinterpret_cast<uintptr_t>(B)) %
+      elem_size(dtype))
+    return BQR_ERR_MISALIGNED;
+  // factor [A | B] (Q^H B falls out of the factorisation) ...
+  int st = bqr_geqrf_qhb_batched(dtype, m, n, nrhs, batch, A, lda, tau, B, ldb, stream);
+  if (st != BQR_SUCCESS) return st;
+  // ... then the triangular system by row operations
+  return solve_upper_dispatch(dtype, A, lda, (long long)lda * n, B, ldb, (long long)ldb * nrhs, info, batch, n,
+                              nrhs, stream);
 }
 
 int bqr_orgqr_batched(bqr_dtype_t dtype, int m, int n, int k, int batch, void *A, int lda,

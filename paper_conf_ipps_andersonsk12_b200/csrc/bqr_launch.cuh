@@ -184,6 +184,9 @@ Plan tiny_plan_c64(int m, int n);
 int apply_dispatch_f32(const ApplyArgs &a, cudaStream_t s);
 int apply_dispatch_c64(const ApplyArgs &a, cudaStream_t s);
 int launch_selftest_math(long long n, unsigned seed, unsigned long long *counts, cudaStream_t s);
+// back substitution X = R^{-1} C of the least-squares path (bqr_solve.cu)
+int solve_upper_dispatch(bqr_dtype_t dt, const void *A, int lda, long long strideA, void *B, int ldb,
+                         long long strideB, int *info, long long batch, int n, int nrhs, cudaStream_t s);
 
 }  // namespace host
 }  // namespace bqr

@@ -719,20 +719,16 @@ struct RfKernel {
   }
 
   // ------------------------------------------------------------ staging
-  // matrix index of this group (recomputed where needed: keeping it in the
-  // context costs two registers through the whole factorisation)
-  static __device__ __forceinline__ long long c_mat(const RfArgs &p, const Ctx &c) {
-    const long long mat = (long long)blockIdx.x * GPB + c.grp;
-    return mat < p.batch ? mat : p.batch - 1;
-  }
-
   // in-bounds test; compile-time true for exact-shape instantiations
   static __device__ __forceinline__ bool inb(int r, int col, int m, int n) {
     if constexpr (EX) return true;
     return r < m && col < n;
   }
 
-  static __device__ __forceinline__ void load_matrix(const RfArgs &p, Ctx &c, float *smem, T *Ab, bool active,
+  // mat: this group's matrix index (the right-hand sides of the augmented
+  // classes live at p.B + mat * strideB)
+  static __device__ __forceinline__ void load_matrix(const RfArgs &p, Ctx &c, float *smem, T *Ab, long long mat,
+                                                     bool active,
                                                      T (&a)[MR][NC]) {
     const int m = p.m, n = p.n;
     if constexpr (STAGE) {
@@ -784,7 +780,7 @@ struct RfKernel {
           a[i][j] = (inb(r, col, m, n) && (EX || active)) ? tile[r + col * ld] : 0.f;
         }
     } else {
-      const T *Bb = reinterpret_cast<const T *>(p.B) + c_mat(p, c) * p.strideB;
+      const T *Bb = reinterpret_cast<const T *>(p.B) + mat * p.strideB;
 #pragma unroll
       for (int i = 0; i < MR; ++i)
 #pragma unroll
@@ -803,7 +799,8 @@ struct RfKernel {
     return x;
   }
 
-  static __device__ __forceinline__ void store_matrix(const RfArgs &p, Ctx &c, float *smem, T *Ab, bool active,
+  static __device__ __forceinline__ void store_matrix(const RfArgs &p, Ctx &c, float *smem, T *Ab, long long mat,
+                                                      bool active,
                                                       const T (&a)[MR][NC]) {
     // opaque reads: keeps ptxas from hoisting the store's per-element
     // predicates above the factorisation loop (they would stay live in
@@ -852,7 +849,7 @@ struct RfKernel {
         }
       }
     } else if (active) {
-      T *Bb = reinterpret_cast<T *>(p.B) + c_mat(p, c) * p.strideB;
+      T *Bb = reinterpret_cast<T *>(p.B) + mat * p.strideB;
 #pragma unroll
       for (int i = 0; i < MR; ++i)
 #pragma unroll
@@ -922,7 +919,7 @@ struct RfKernel {
             }
         }
       } else {
-        load_matrix(p, c, smem, Ab, true, a);
+        load_matrix(p, c, smem, Ab, mat, true, a);
       }
       __syncthreads();  // tile consumed by every thread
       const long long nxt = mat + gridDim.x;
@@ -936,7 +933,7 @@ struct RfKernel {
       c.dbg = false;
 #endif
       __syncthreads();  // every tau published before the tau store
-      store_matrix(p, c, smem, Ab, true, a);
+      store_matrix(p, c, smem, Ab, mat, true, a);
       T *tg = reinterpret_cast<T *>(p.tau) + mat * p.strideT;
       for (int idx = t; idx < p.kmax; idx += GT) tg[idx] = c.taus[idx];
       __syncthreads();  // vector/tau buffers reused by the next matrix
@@ -1094,7 +1091,7 @@ struct RfKernel {
     c.taus = c.vbuf + NBUF * VB;
     T *Ab = reinterpret_cast<T *>(p.A) + mat * p.strideA;
     T a[MR][NC];
-    load_matrix(p, c, smem, Ab, active, a);
+    load_matrix(p, c, smem, Ab, mat, active, a);
 
     if constexpr (ORG) {
       // columns >= k start as the identity (xORG2R initialisation)
@@ -1116,7 +1113,7 @@ struct RfKernel {
       group_sync<GT, GPB>(grp);  // every tau published before the tau store
     }
 
-    store_matrix(p, c, smem, Ab, active, a);
+    store_matrix(p, c, smem, Ab, mat, active, a);
     // tau list -> global (each tau was published before a group barrier)
     if (!ORG && active) {
       T *tg = reinterpret_cast<T *>(p.tau) + mat * p.strideT;

@@ -72,3 +72,20 @@ def geqrf_qhb_gpu(A_cm: np.ndarray, m: int, B_cm: np.ndarray):
     assert st == 0, st
     torch.cuda.synchronize()
     return A.cpu().numpy(), tau.cpu().numpy(), B.cpu().numpy()
+
+
+def gels_gpu(A_cm: np.ndarray, m: int, B_cm: np.ndarray):
+    """Least squares through bqr_gels_batched; returns (A_out_cm, tau, B_out_cm, info)."""
+    import ctypes
+    A = to_dev(A_cm)
+    B = to_dev(B_cm)
+    batch, n, lda = A_cm.shape
+    _, nrhs, ldb = B_cm.shape
+    tau = torch.empty((batch, n), dtype=A.dtype, device="cuda")
+    info = torch.full((batch,), -7, dtype=torch.int32, device="cuda")
+    st = bqr.load().bqr_gels_batched(bqr.R32 if A.dtype == torch.float32 else bqr.C64, m, n, nrhs, batch,
+                                     ctypes.c_void_p(A.data_ptr()), lda, ctypes.c_void_p(tau.data_ptr()),
+                                     ctypes.c_void_p(B.data_ptr()), ldb, ctypes.c_void_p(info.data_ptr()), None)
+    assert st == 0, st
+    torch.cuda.synchronize()
+    return A.cpu().numpy(), tau.cpu().numpy(), B.cpu().numpy(), info.cpu().numpy()

@@ -149,3 +149,25 @@ def test_qhb_argument_checks(lib, args, code):
     st = lib.bqr_geqrf_qhb_batched(d, m, n, nrhs, b, ctypes.c_void_p(A), lda, ctypes.c_void_p(tau),
                                    ctypes.c_void_p(B), ldb, None)
     assert st == code
+
+
+@pytest.mark.parametrize("args,code", [
+    ((7, 8, 4, 1, 1, FAKE, 8, FAKE, FAKE, 8), -1),
+    ((0, -1, 4, 1, 1, FAKE, 8, FAKE, FAKE, 8), -2),
+    ((0, 8, -1, 1, 1, FAKE, 8, FAKE, FAKE, 8), -3),
+    ((0, 8, 4, -1, 1, FAKE, 8, FAKE, FAKE, 8), -4),
+    ((0, 8, 4, 1, -1, FAKE, 8, FAKE, FAKE, 8), -5),
+    ((0, 8, 4, 1, 1, 0, 8, FAKE, FAKE, 8), -6),
+    ((0, 8, 4, 1, 1, FAKE, 7, FAKE, FAKE, 8), -7),
+    ((0, 8, 4, 1, 1, FAKE, 8, 0, FAKE, 8), -8),
+    ((0, 8, 4, 1, 1, FAKE, 8, FAKE, 0, 8), -9),
+    ((0, 8, 4, 1, 1, FAKE, 8, FAKE, FAKE, 7), -10),
+    ((0, 8, 4, 1, 0, 0, 8, 0, 0, 8), 0),              # batch == 0: quick return
+    ((0, 4, 8, 1, 1, FAKE, 4, FAKE, FAKE, 4), 1),     # m < n (minimum norm): not supported
+    ((0, 8, 4, 1, 1, FAKE + 2, 8, FAKE, FAKE, 8), 3),  # misaligned
+])
+def test_gels_argument_checks(lib, args, code):
+    d, m, n, nrhs, b, A, lda, tau, B, ldb = args
+    st = lib.bqr_gels_batched(d, m, n, nrhs, b, ctypes.c_void_p(A), lda, ctypes.c_void_p(tau), ctypes.c_void_p(B),
+                              ldb, None, None)
+    assert st == code

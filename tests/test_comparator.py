@@ -136,3 +136,47 @@ def test_accepts_cascade_after_tie_flip():
     out_cm = oracle.to_cm(R[None].astype(np.float32))
     rep = compare_geqrf(A_cm, m, out_cm, np.array([taus], dtype=np.float32))
     assert rep["flips"] >= 1 and rep["ok"], rep
+
+
+# ---------------------------------------------------------------- gels
+def _ls_problem(m, n, cplx, seed=0, batch=3):
+    rng = np.random.default_rng(seed)
+    A = rng.standard_normal((batch, m, n))
+    B = rng.standard_normal((batch, m, 1))
+    if cplx:
+        A = A + 1j * rng.standard_normal((batch, m, n))
+        B = B + 1j * rng.standard_normal((batch, m, 1))
+    dt = np.complex64 if cplx else np.float32
+    return oracle.to_cm(A.astype(dt)), oracle.to_cm(B.astype(dt))
+
+
+@pytest.mark.parametrize("m,n,cplx", [(240, 66, True), (56, 56, False), (80, 16, True)])
+def test_compare_gels_accepts_fp32_lapack(m, n, cplx):
+    """Single-precision LAPACK xGELS output passes the comparator."""
+    import scipy.linalg.lapack as L
+    from oracle.compare import compare_gels
+    A_cm, B_cm = _ls_problem(m, n, cplx)
+    Bout = B_cm.copy()
+    fn = L.cgels if cplx else L.sgels
+    for b in range(A_cm.shape[0]):
+        A = oracle.from_cm(A_cm[b:b + 1], m)[0]
+        bb = oracle.from_cm(B_cm[b:b + 1], m)[0]
+        res = fn(A.copy(), bb.copy())
+        Bout[b] = oracle.to_cm(res[1][None])[0]
+    rep = compare_gels(A_cm, m, B_cm, Bout, np.zeros(A_cm.shape[0], np.int32))
+    assert rep["ok"], rep
+
+
+def test_compare_gels_rejects_wrong_solutions():
+    from oracle.compare import compare_gels
+    A_cm, B_cm = _ls_problem(240, 66, True)
+    _, _, Bo, info = oracle.gels_cm(A_cm, 240, B_cm)
+    good = Bo.astype(np.complex64)
+    assert compare_gels(A_cm, 240, B_cm, good, info)["ok"]
+    bad = good.copy()
+    bad[0, 0, 5] *= 1.001  # one solution entry off by 1e-3 relative
+    assert not compare_gels(A_cm, 240, B_cm, bad, info)["ok"]
+    conj = good.copy()
+    conj[:, :, :66] = np.conj(conj[:, :, :66])  # a dropped conjugate
+    assert not compare_gels(A_cm, 240, B_cm, conj, info)["ok"]
+    assert not compare_gels(A_cm, 240, B_cm, good, info + 1)["ok"]  # wrong info

@@ -226,6 +226,19 @@ def test_fused_geqrf_qhb(dt, m, n, nrhs):
     assert r["ok"], r
 
 
+def test_fused_stap_full_batch_persistent_loop():
+    """The bench's C4 step: 256 STAP matrices, more than one per CTA of the
+    persistent loop (regression: the right-hand sides of a CTA's second
+    matrix were stored into its first matrix's slot)."""
+    A = bqr_inputs.config_batch("C4")
+    B = bqr_inputs.rhs_batch(240, 1, 256, "c64", seed=4)
+    out, tau, QhB = geqrf_qhb_gpu(A, 240, B)
+    rep = compare_geqrf(A, 240, out, tau, full_q=False)
+    assert rep["ok"], rep
+    r = compare_apply(out, 240, 66, tau, B, QhB)
+    assert r["ok"], r
+
+
 def test_fused_stap_is_one_kernel():
     import paper_conf_ipps_andersonsk12_b200 as bqr
     assert bqr.load().bqr_qhb_kernel_name(bqr.C64, 240, 66, 1).decode().startswith("rf_c64")
