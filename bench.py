@@ -193,6 +193,10 @@ def max_over_ranks(torch, dist, world, x: float) -> float:
     return bqr_dist.max_over_ranks(torch, dist, x)
 
 
+# context only (another machine): the paper's Table VII GPU GFLOP/s
+PAPER_TABLE_VII = {"S80": 134.0, "S192": 98.0}
+
+
 def time_workload(w: Workload, steps: int, warmup: int, torch, dist, world, flush, sampler=None, fused=True):
     """Returns (ms_per_step, ms_of_the_factorisation_kernel).  With right-hand
     sides the step is the fused factorisation + Q^H b (one kernel, the
@@ -363,7 +367,7 @@ def run_ours(args):
     out["gpu_launches"] += (e_steps + 2) * 0  # e2e launches are outside the device-timed kernel region
     if not args.no_also:
         also = {}
-        for name in [c for c in ("C4", "C2") if c != args.config]:
+        for name in [c for c in ("C4", "C2", "S80", "S192") if c != args.config]:
             w = Workload(name, rank, world, torch, bqr)
             k2 = max(3, min(args.steps, 100))
             s_ms, q_ms = time_workload(w, k2, max(3, args.warmup), torch, dist, world, flush)
@@ -373,6 +377,8 @@ def run_ours(args):
                           "matrices_per_s": round(world * w.batch / (s_ms / 1e3), 1),
                           "config": config_block(w, world, l2_note),
                           "roofline": roofline_obj(w, q_ms, peaks, n_sm, fused=bool(w.nrhs))}
+            if name in PAPER_TABLE_VII:
+                also[name]["paper_quadro6000_gflops"] = PAPER_TABLE_VII[name]
             out["gpu_launches"] += k2
             if w.nrhs:
                 # context: the same step as two launches (geqrf, then apply_qh)
@@ -435,7 +441,7 @@ def main():
     ap.add_argument("--steps", type=int, default=200)
     ap.add_argument("--warmup", type=int, default=10)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--config", default="C3", choices=["C1", "C2", "C3", "C4"])
+    ap.add_argument("--config", default="C3", choices=["C1", "C2", "C3", "C4", "S80", "S192"])
     ap.add_argument("--no-also", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     args = ap.parse_args()

@@ -31,6 +31,10 @@ CONFIGS = {
     "C2": dict(m=4, n=4, batch=1_000_000, dtype="f32", dist="uniform", seed=2),
     "C3": dict(m=56, n=56, batch=5000, dtype="f32", dist="normal", seed=3),
     "C4": dict(m=240, n=66, batch=256, dtype="c64", dist="normal", seed=4, nrhs=1),
+    # NEXT-2: the paper's other RT_STAP sizes (Table VII, P:L1113-1123:
+    # "80x16 384", "192x96 128"; complex single precision, QR only)
+    "S80": dict(m=80, n=16, batch=384, dtype="c64", dist="normal", seed=5),
+    "S192": dict(m=192, n=96, batch=128, dtype="c64", dist="normal", seed=6),
 }
 
 

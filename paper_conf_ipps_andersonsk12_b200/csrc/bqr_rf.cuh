@@ -193,11 +193,24 @@ struct RfCfg {
   static constexpr int MRP = mrp_calc();
   static constexpr int VB = R * MRP;          // elements per vector buffer
   // multi-warp groups publish ahead without a full barrier (see step_arrive)
-  static constexpr int NBUF = GT <= 32 ? 2 : 32 / R + 2;
+  // lazy rest-update (see RfKernel::step): one column group per warp only
+#ifndef BQR_LAZY
+#define BQR_LAZY 1
+#endif
+  static constexpr bool LAZY = BQR_LAZY != 0 && GT > 32 && R == 32 && !STAGE;
+  // Lazy groups are also decoupled: the publishing warp signals a "full"
+  // mbarrier per vector buffer and a consumer waits only for that producer
+  // (a named barrier with the group's thread count made every step a
+  // rendezvous of all warps).  There is no consumer -> producer signal:
+  // when v_j is published, every warp w has published its column c in
+  // [j-G, j-1] and may still read only v_{c-2} or later, so G + 3 buffers
+  // are never overwritten while read.
+  static constexpr int NBUF = GT <= 32 ? 2 : (LAZY ? G + 3 : 32 / R + 2);
   static_assert(GT <= 32 || GPB == 1, "multi-warp groups: one group per CTA");
   // [NBUF][VB] vectors | [NMAX] taus | mbarrier (8-byte aligned, 4 words)
   static constexpr int kMbarWord = ((NBUF * VB + NMAX) * E + 3) / 4 * 4;
-  static constexpr int kSmallWords = kMbarWord + 4;
+  static constexpr int kFullWord = kMbarWord + 4;  // LAZY: [NBUF] "full" mbarriers
+  static constexpr int kSmallWords = kFullWord + (LAZY ? 2 * NBUF : 0);
   static constexpr int kSmallAll = ((GPB * kSmallWords + 31) / 32) * 32;
   static_assert(R >= 1 && R <= 32 && (R & (R - 1)) == 0, "R must be a power of two <= 32");
   static_assert(GT <= 32 ? (32 % GT == 0) : (GT % 32 == 0 && 32 % R == 0), "group must tile warps");
@@ -228,6 +241,8 @@ struct RfKernel {
     int rg, cg, t, lane, grp;
     int wid;   // warp index in the group, warp-uniform by construction (shfl)
     int kmax;
+    unsigned long long *full;  // LAZY: [NBUF] full barriers
+    int gbase;                 // LAZY: steps published before this matrix
 #ifdef BQR_PHASE_TIMING
     bool dbg;
 #endif
@@ -238,6 +253,29 @@ struct RfKernel {
     T scal, tau;
     float beta;
   };
+
+  // ------------------------------------------------------------ step signals
+  static __device__ __forceinline__ void sig_arrive(Ctx &c, int k) {
+    if constexpr (Cfg::LAZY) {
+      // every lane of the publishing warp arrives (count 32): each lane's
+      // vector stores are released by its own arrive
+      asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(c.full + (c.gbase + k) % NBUF))
+                   : "memory");
+    } else {
+      step_arrive<GT, NBUF>(k);
+    }
+  }
+  static __device__ __forceinline__ void sig_wait(Ctx &c, int k) {
+    if constexpr (Cfg::LAZY) {
+      const int g = c.gbase + k;
+      void *b = c.full + g % NBUF;
+      const unsigned par = (unsigned)(g / NBUF) & 1u;
+      while (!mbar_try_wait(b, par)) {
+      }
+    } else {
+      step_wait<GT, NBUF>(k);
+    }
+  }
 
   // ------------------------------------------------------------ smem vector I/O
   // load rows [I0, MR) of this lane's Householder vector (others left unset)
@@ -373,13 +411,168 @@ struct RfKernel {
     }
   }
 
+  // ------------------------------------------------------------ packed FP32 (FFMA2)
+  // sm_100a issues a packed fp32x2 FMA (fma.rn.f32x2, SASS FFMA2) per lane in
+  // one slot: the same IEEE fma on two operand pairs.  The kernels are issue
+  // bound (ncu: IPC ~1.9 of 4, FFMA ~53% of the instructions), so the
+  // matrix-vector product and the rank-1 update run on row pairs (real) or
+  // on the (re, im) pair (complex), halving the FMA issue slots.
+#ifndef BQR_FFMA2
+#define BQR_FFMA2 1
+#endif
+  // real classes with the largest register tiles (C3's 14x14 per lane) lose
+  // more to register-pair moves and spills than they gain (measured)
+  static constexpr bool kPacked = BQR_FFMA2 != 0 && (X::kComplex || MR * NC <= 128);
+
+  static __device__ __forceinline__ float2 pk(float x, float y) { return make_float2(x, y); }
+
+  // Real: H_k applied to slots [J0, J1) with rows paired (2p, 2p+1); a leading
+  // odd row I0 and a trailing odd row MR-1 run as scalar FMAs.  Each product
+  // is the same fma as the scalar path; only the summation grouping of the
+  // dot products differs (two interleaved partial sums per accumulator).
+  template <int P, int I0, int J0, int J1>
+  static __device__ __forceinline__ void apply_pk_real(Ctx &c, float (&a)[MR][NC], const float *vb, float ct, int kk) {
+    constexpr int NS = J1 - J0;
+    constexpr int IP = (I0 + 1) & ~1;
+    constexpr int NPR = (MR - IP) / 2;
+    constexpr bool HEAD = IP > I0 && I0 < MR;
+    constexpr bool TAIL = ((MR - IP) & 1) != 0 && IP < MR;
+    constexpr int ACC = NS <= 6 ? 2 : 1;
+    float2 w2[NS][ACC];
+    float ws[NS];
+#pragma unroll
+    for (int j = 0; j < NS; ++j) {
+      ws[j] = 0.f;
+#pragma unroll
+      for (int q = 0; q < ACC; ++q) w2[j][q] = pk(0.f, 0.f);
+    }
+    {
+      float v[MR];
+      load_v<I0>(vb, v);
+#pragma unroll
+      for (int p = 0; p < NPR; ++p) {
+        const int i = IP + 2 * p;
+        const float2 v2 = pk(v[i], v[i + 1]);
+#pragma unroll
+        for (int j = 0; j < NS; ++j)
+          w2[j][p % ACC] = __ffma2_rn(v2, pk(a[i][J0 + j], a[i + 1][J0 + j]), w2[j][p % ACC]);
+      }
+#pragma unroll
+      for (int j = 0; j < NS; ++j) {
+        if constexpr (HEAD) ws[j] = fmaf(v[I0], a[I0][J0 + j], ws[j]);
+        if constexpr (TAIL) ws[j] = fmaf(v[MR - 1], a[MR - 1][J0 + j], ws[j]);
+      }
+    }
+    float sum[NS];
+#pragma unroll
+    for (int j = 0; j < NS; ++j) {
+      float2 s2 = w2[j][0];
+      if constexpr (ACC == 2) s2 = __fadd2_rn(s2, w2[j][1]);
+      sum[j] = (s2.x + s2.y) + ws[j];
+    }
+    if constexpr (R >= 8 && NS >= 2) {
+      row_allreduce_multi<R, NS>(sum, c.lane);
+    } else {
+#pragma unroll
+      for (int j = 0; j < NS; ++j) sum[j] = row_allreduce<R>(sum[j]);
+    }
+    float tw[NS];
+#pragma unroll
+    for (int j = 0; j < NS; ++j) {
+      tw[j] = ct * sum[j];
+      if (J0 + j == P) tw[j] = c.cg > kk ? tw[j] : 0.f;
+    }
+    {
+      float v[MR];
+      load_v<I0>(vb, v);
+#pragma unroll
+      for (int j = 0; j < NS; ++j) {
+        const float2 nt = pk(-tw[j], -tw[j]);
+#pragma unroll
+        for (int p = 0; p < NPR; ++p) {
+          const int i = IP + 2 * p;
+          const float2 r = __ffma2_rn(pk(v[i], v[i + 1]), nt, pk(a[i][J0 + j], a[i + 1][J0 + j]));
+          a[i][J0 + j] = r.x;
+          a[i + 1][J0 + j] = r.y;
+        }
+        if constexpr (HEAD) a[I0][J0 + j] = fmaf(-v[I0], tw[j], a[I0][J0 + j]);
+        if constexpr (TAIL) a[MR - 1][J0 + j] = fmaf(-v[MR - 1], tw[j], a[MR - 1][J0 + j]);
+      }
+    }
+  }
+
+  // Complex: conj(v) a = (vr, vr) * (ar, ai) + (vi, vi) * (ar, ai) recombined
+  // as (A.x + B.y, A.y - B.x); the update a -= v t is
+  // a = fma2((vr, vr), (-tr, -ti), a); a = fma2((vi, vi), (ti, -tr), a).
+  template <int P, int I0, int J0, int J1>
+  static __device__ __forceinline__ void apply_pk_cplx(Ctx &c, float2 (&a)[MR][NC], const float2 *vb, float2 ct,
+                                                      int kk) {
+    constexpr int NS = J1 - J0;
+    float2 wa[NS], wb[NS];
+#pragma unroll
+    for (int j = 0; j < NS; ++j) wa[j] = wb[j] = pk(0.f, 0.f);
+    {
+      float2 v[MR];
+      load_v<I0>(vb, v);
+#pragma unroll
+      for (int i = I0; i < MR; ++i) {
+        const float2 vr = pk(v[i].x, v[i].x), vi = pk(v[i].y, v[i].y);
+#pragma unroll
+        for (int j = 0; j < NS; ++j) {
+          wa[j] = __ffma2_rn(vr, a[i][J0 + j], wa[j]);
+          wb[j] = __ffma2_rn(vi, a[i][J0 + j], wb[j]);
+        }
+      }
+    }
+    float f[2 * NS];
+#pragma unroll
+    for (int j = 0; j < NS; ++j) {
+      f[2 * j] = wa[j].x + wb[j].y;
+      f[2 * j + 1] = wa[j].y - wb[j].x;
+    }
+    if constexpr (R >= 8) {
+      row_allreduce_multi<R, 2 * NS>(f, c.lane);
+    } else {
+#pragma unroll
+      for (int q = 0; q < 2 * NS; ++q) f[q] = row_allreduce_f<R>(f[q]);
+    }
+    float2 n1[NS], n2[NS];
+#pragma unroll
+    for (int j = 0; j < NS; ++j) {
+      float2 t = X::mul(ct, pk(f[2 * j], f[2 * j + 1]));
+      if (J0 + j == P) t = X::sel(c.cg > kk, t, X::zero());
+      n1[j] = pk(-t.x, -t.y);
+      n2[j] = pk(t.y, -t.x);
+    }
+    {
+      float2 v[MR];
+      load_v<I0>(vb, v);
+#pragma unroll
+      for (int i = I0; i < MR; ++i) {
+        const float2 vr = pk(v[i].x, v[i].x), vi = pk(v[i].y, v[i].y);
+#pragma unroll
+        for (int j = 0; j < NS; ++j) a[i][J0 + j] = __ffma2_rn(vi, n2[j], __ffma2_rn(vr, n1[j], a[i][J0 + j]));
+      }
+    }
+  }
+
+  template <int P, int I0, int J0, int J1>
+  static __device__ __forceinline__ void apply_pk(Ctx &c, T (&a)[MR][NC], const T *vb, T ct, int kk) {
+    if constexpr (X::kComplex)
+      apply_pk_cplx<P, I0, J0, J1>(c, a, vb, ct, kk);
+    else
+      apply_pk_real<P, I0, J0, J1>(c, a, vb, ct, kk);
+  }
+
   // ------------------------------------------------------------ trailing update
   // Apply H_k^H (vector in vb, conj(tau) = ct) to slots [J0, J1); slot P
   // columns with cg <= kk are excluded (already factored).  The vector is
   // re-read from shared memory in 16-byte chunks for each pass.
   template <int P, int I0, int J0, int J1>
   static __device__ __forceinline__ void apply(Ctx &c, T (&a)[MR][NC], const T *vb, T ct, int kk) {
-    if constexpr (J0 < J1) {
+    if constexpr (kPacked && J0 < J1) {
+      apply_pk<P, I0, J0, J1>(c, a, vb, ct, kk);
+    } else if constexpr (J0 < J1) {
       constexpr int NS = J1 - J0;
       // partial sums per slot: ptxas walks the slots one after another, so a
       // single accumulator per slot is a 4-cycle-per-row serial chain; 4 is
@@ -447,7 +640,7 @@ struct RfKernel {
     if (warp_has(c, k)) {
       const Look l = reflector<P, I0>(c, a, k);
       publish<P, I0>(c, a, k, l, true);
-      step_arrive<GT, NBUF>(k);
+      sig_arrive(c, k);
     }
   }
 
@@ -458,7 +651,7 @@ struct RfKernel {
   static __device__ __forceinline__ void step(Ctx &c, T (&a)[MR][NC], int k) {
     const int kk = k - P * G;
     BQR_STAMP(c, k, 0);
-    if (!warp_has(c, k) || GT <= 32) step_wait<GT, NBUF>(k);
+    if (!warp_has(c, k) || GT <= 32) sig_wait(c, k);
     BQR_STAMP(c, k, 1);
     const T ct = X::conj(c.taus[k]);
     const T *vb = c.vbuf + buf(k) * VB + c.rg * MRP;
@@ -473,14 +666,26 @@ struct RfKernel {
       publish<P, I0>(c, a, k + 1, l, la);
       BQR_STAMP(c, k, 3);
     } else {
-      // multi-warp groups: publish first so the other warps never wait
+      // multi-warp groups: publish first so the other warps never wait.
+      // Lazy rest-update: the warp that will own column k+2 applies H_k only
+      // to its slot P here and defers the other slots to step k+1, after it
+      // has published v_{k+2}; otherwise its whole rest-update of step k
+      // sits between v_{k+1} arriving and the reflector chain of column k+2
+      // (ncu: 15% of warp time in barrier stalls waiting for that chain).
+      const bool defer = Cfg::LAZY && kk + 2 < G && k + 2 < c.kmax && warp_has(c, k + 2);
+      const bool catchup = Cfg::LAZY && la && kk >= 1;
       if (la) {
         const Look l = reflector<P, I0>(c, a, k + 1);
         publish<P, I0>(c, a, k + 1, l, true);
-        step_arrive<GT, NBUF>(k + 1);
+        sig_arrive(c, k + 1);
       }
       BQR_STAMP(c, k, 2);
-      apply<P, I0, P + 1, NC>(c, a, vb, ct, kk);
+      if (catchup) {
+        const T ctp = X::conj(c.taus[k - 1]);
+        const T *vbp = c.vbuf + buf(k - 1) * VB + c.rg * MRP;
+        apply<P, I0, P + 1, NC>(c, a, vbp, ctp, kk - 1);
+      }
+      if (!defer) apply<P, I0, P + 1, NC>(c, a, vb, ct, kk);
       BQR_STAMP(c, k, 3);
     }
   }
@@ -887,8 +1092,14 @@ struct RfKernel {
     T *tile = reinterpret_cast<T *>(smem + Cfg::kSmallAll);
     void *bar = smem + Cfg::kMbarWord;
     const int m = p.m, n = p.n;
-    if (p.bulk) {
-      if (t == 0) mbar_init(bar, 1);
+    c.full = reinterpret_cast<unsigned long long *>(smem + Cfg::kFullWord);
+    c.gbase = 0;
+    if (p.bulk || Cfg::LAZY) {
+      if (t == 0) {
+        if (p.bulk) mbar_init(bar, 1);
+        if constexpr (Cfg::LAZY)
+          for (int b = 0; b < NBUF; ++b) mbar_init(c.full + b, 32);
+      }
       __syncthreads();
     }
     bool have_tile = false;
@@ -937,6 +1148,7 @@ struct RfKernel {
       T *tg = reinterpret_cast<T *>(p.tau) + mat * p.strideT;
       for (int idx = t; idx < p.kmax; idx += GT) tg[idx] = c.taus[idx];
       __syncthreads();  // vector/tau buffers reused by the next matrix
+      c.gbase += p.kmax;
     }
   }
 

@@ -53,6 +53,16 @@ def test_C3_56x56_full():
     assert rep["residual_max"] < 2e-6 and rep["orth_max"] < 5e-6
 
 
+@pytest.mark.parametrize("name", ["S80", "S192"])
+def test_stap_table_vii_full(name):
+    """NEXT-2: the paper's other RT_STAP QR sizes (Table VII),
+    full batch in the bench's launch configuration."""
+    A = bqr_inputs.config_batch(name)
+    m = bqr_inputs.CONFIGS[name]["m"]
+    _, _, rep = _check(A, m, full_q=False)
+    assert rep["residual_max"] < 2e-6
+
+
 def test_C4_stap_240x66_full_with_apply():
     A = bqr_inputs.config_batch("C4")
     out, tau, rep = _check(A, 240, full_q=False)
