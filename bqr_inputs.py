@@ -96,6 +96,30 @@ def random_batch(m: int, n: int, batch: int, dtype: str = "f32", seed: int = 0,
     return out
 
 
+def diag_dominant_batch(n: int, batch: int, dtype: str = "f32", seed: int = 0,
+                        lda: int | None = None, start: int = 0,
+                        stop: int | None = None) -> np.ndarray:
+    """NEXT-3 inputs (LU / Gauss-Jordan without pivoting): the paper ran them
+    on "diagonally-dominant matrices so no pivoting was necessary"
+    (P:L1009).  Off-diagonal entries are the seeded iid Gaussian
+    stream of random_batch; each diagonal entry is replaced by
+    +-(1 + max(column sum, row sum) of the off-diagonal magnitudes), so the
+    matrix is strictly diagonally dominant by rows and by columns (the sign
+    is the sign of the original draw).  Column-major (batch', n, lda)."""
+    A = random_batch(n, n, batch, dtype, seed, "normal", lda=lda, start=start, stop=stop)
+    lda = n if lda is None else lda
+    core = A[:, :, :n]
+    mag = np.abs(core).astype(np.float64)
+    idx = np.arange(n)
+    diag_mag = mag[:, idx, idx]
+    colsum = mag.sum(axis=2) - diag_mag   # storage [b, col, row]: sum over rows
+    rowsum = mag.sum(axis=1) - diag_mag
+    d = 1.0 + np.maximum(colsum, rowsum)
+    sgn = np.where(np.real(core[:, idx, idx]) < 0, -1.0, 1.0)
+    core[:, idx, idx] = (sgn * d).astype(core.dtype)
+    return A
+
+
 def config_batch(name: str, start: int = 0, stop: int | None = None,
                  batch: int | None = None) -> np.ndarray:
     cfg = CONFIGS[name]

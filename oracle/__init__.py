@@ -31,6 +31,7 @@ import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
 _SRC = os.path.join(_HERE, "bqr_ref.c")
+_SRCS = [_SRC, os.path.join(_HERE, "lu_ref.c")]  # lu_ref.c: NEXT-3 (LU / Gauss-Jordan)
 _LIB = os.path.join(_HERE, "libbqr_ref.so")
 _lock = threading.Lock()
 _lib = None
@@ -38,9 +39,9 @@ _lib = None
 
 def build(force: bool = False) -> str:
     """Compile libbqr_ref.so with gcc -O2 -fopenmp (no -ffast-math: IEEE fp64)."""
-    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
+    if force or not os.path.exists(_LIB) or any(os.path.getmtime(_LIB) < os.path.getmtime(s) for s in _SRCS):
         cmd = ["gcc", "-O2", "-std=c11", "-fopenmp", "-fPIC", "-shared",
-               "-fno-fast-math", "-ffp-contract=off", "-o", _LIB, _SRC, "-lm"]
+               "-fno-fast-math", "-ffp-contract=off", "-o", _LIB, *_SRCS, "-lm"]
         subprocess.check_call(cmd)
     return _LIB
 
@@ -63,6 +64,12 @@ def _load():
                 getattr(lib, name).restype = None
             for name in ("bqr_ref_gels_d", "bqr_ref_gels_z"):
                 getattr(lib, name).argtypes = [i, i, i, i64, p, i, p, p, i, p]
+                getattr(lib, name).restype = None
+            for name in ("bqr_ref_getrf_np_d", "bqr_ref_getrf_np_z"):
+                getattr(lib, name).argtypes = [i, i, i64, p, i, p]
+                getattr(lib, name).restype = None
+            for name in ("bqr_ref_gauss_jordan_d", "bqr_ref_gauss_jordan_z"):
+                getattr(lib, name).argtypes = [i, i, i64, p, i, p, i, p]
                 getattr(lib, name).restype = None
             lib.bqr_ref_set_threads.argtypes = [i]
             lib.bqr_ref_max_threads.restype = i
@@ -216,3 +223,59 @@ def gels(A: np.ndarray, B: np.ndarray):
     Bl = from_cm(Bo, m)
     return Bl[:, :n, :], Bl[:, n:, :], info
 
+
+
+# ---------------------------------------------------------------- NEXT-3
+# LU without pivoting and Gauss-Jordan (paper Sec. III-A/B, P:L267-275,
+# Listings 5-7); arithmetic in lu_ref.c.
+
+def getrf_np_cm(A_cm: np.ndarray, m: int):
+    """LU without pivoting on column-major storage A (batch, n, lda).
+    Returns (LU_cm: L strictly lower (unit diagonal implied) + U upper,
+    info (batch,) int32: 0 or k+1 for the first zero pivot)."""
+    lib = _load()
+    A = _widen(A_cm).copy()
+    batch, n, lda = A.shape
+    info = np.zeros((batch,), dtype=np.int32)
+    if batch and m and n:
+        fn = lib.bqr_ref_getrf_np_z if _is_complex(A) else lib.bqr_ref_getrf_np_d
+        fn(m, n, batch, _ptr(A), lda, _ptr(info))
+    return A, info
+
+
+def getrf_np(A: np.ndarray):
+    """Logical API: A (batch, m, n) -> (LU (batch, m, n), info)."""
+    A = np.asarray(A)
+    if A.ndim == 2:
+        A = A[None]
+    m = A.shape[1]
+    LU, info = getrf_np_cm(to_cm(A), m)
+    return from_cm(LU, m), info
+
+
+def gauss_jordan_cm(A_cm: np.ndarray, B_cm: np.ndarray):
+    """Gauss-Jordan on [A | B] without pivoting, column-major storage:
+    A (batch, n, lda) with n x n matrices, B (batch, nrhs, ldb).  Returns
+    (A_out_cm, X_cm, info): X overwrites B; A keeps the multipliers
+    off the diagonal and pivot * (1/pivot) on it (lu_ref.c, reading L2)."""
+    lib = _load()
+    A = _widen(A_cm).copy()
+    batch, n, lda = A.shape
+    B = np.ascontiguousarray(B_cm, dtype=A.dtype).copy()
+    _, nrhs, ldb = B.shape
+    info = np.zeros((batch,), dtype=np.int32)
+    if batch and n:
+        fn = lib.bqr_ref_gauss_jordan_z if _is_complex(A) else lib.bqr_ref_gauss_jordan_d
+        fn(n, nrhs, batch, _ptr(A), lda, _ptr(B), ldb, _ptr(info))
+    return A, B, info
+
+
+def gauss_jordan(A: np.ndarray, B: np.ndarray):
+    """Logical API: A (batch, n, n), B (batch, n, nrhs) -> (X, info)."""
+    A = np.asarray(A)
+    B = np.asarray(B)
+    if A.ndim == 2:
+        A, B = A[None], B[None]
+    n = A.shape[1]
+    _, X, info = gauss_jordan_cm(to_cm(A), to_cm(B))
+    return from_cm(X, n), info
