@@ -129,8 +129,8 @@ class Workload:
         self.torch, self.bqr = torch, bqr
         # weak scaling: rank r owns matrices [r*B, (r+1)*B) of a world*B seeded stream
         lo, hi = bqr_dist.rank_slice(rank, world, self.batch)
-        host = bqr_inputs.random_batch(self.m, self.n, world * self.batch, self.dt, cfg["seed"], cfg["dist"],
-                                       start=lo, stop=hi)
+        self.kind = cfg.get("kind", "qr")
+        host = bqr_inputs.config_batch(name, start=lo, stop=hi, batch=world * self.batch)
         self.host = host
         self.pristine = torch.from_numpy(host).cuda()
         self.A = torch.empty_like(self.pristine)
@@ -149,7 +149,16 @@ class Workload:
         self.c = ctypes
         self.flops = self.batch * bm.geqrf_flops(self.m, self.n, self.dt)
         self.bytes = self.batch * bm.geqrf_bytes(self.m, self.n, self.dt)
-        if self.nrhs:
+        if self.kind != "qr":  # NEXT-3: LU / Gauss-Jordan
+            self.info = torch.empty((self.batch,), dtype=torch.int32, device="cuda")
+            if self.kind == "lu":
+                self.flops = self.batch * bm.lu_flops(self.m, self.n, self.dt)
+                self.bytes = self.batch * bm.lu_bytes(self.m, self.n, self.dt)
+            else:
+                self.flops = self.batch * bm.gj_flops(self.n, self.dt)
+                self.bytes = self.batch * bm.gj_bytes(self.n, self.nrhs, self.dt)
+            self.flops_apply = self.bytes_apply = 0
+        elif self.nrhs:
             self.flops_apply = self.batch * bm.apply_flops(self.m, self.n, self.nrhs, self.dt)
             self.bytes_apply = self.batch * bm.apply_bytes(self.m, self.nrhs, self.dt)
         else:
@@ -162,6 +171,19 @@ class Workload:
 
     def geqrf(self):
         c = self.c
+        if self.kind == "lu":
+            st = self.lib.bqr_getrf_np_batched(self.code, self.m, self.n, self.batch, c.c_void_p(self.A.data_ptr()),
+                                               self.m, c.c_void_p(self.info.data_ptr()), c.c_void_p(self.sptr))
+            if st:
+                raise RuntimeError(f"bqr_getrf_np_batched -> {st}")
+            return
+        if self.kind == "gj":
+            st = self.lib.bqr_gauss_jordan_batched(self.code, self.n, self.nrhs, self.batch,
+                                                   c.c_void_p(self.A.data_ptr()), self.n, c.c_void_p(self.B.data_ptr()),
+                                                   self.n, c.c_void_p(self.info.data_ptr()), c.c_void_p(self.sptr))
+            if st:
+                raise RuntimeError(f"bqr_gauss_jordan_batched -> {st}")
+            return
         st = self.lib.bqr_geqrf_batched(self.code, self.m, self.n, self.batch, c.c_void_p(self.A.data_ptr()),
                                         self.m, c.c_void_p(self.tau.data_ptr()), c.c_void_p(self.sptr))
         if st:
@@ -206,7 +228,7 @@ def time_workload(w: Workload, steps: int, warmup: int, torch, dist, world, flus
     def run_step(i=None):
         if i is not None:
             ev[i][0].record(w.stream)
-        if w.nrhs and fused:
+        if w.nrhs and fused and w.kind == "qr":
             w.geqrf_qhb()
             if i is not None:
                 ev[i][1].record(w.stream)
@@ -214,7 +236,7 @@ def time_workload(w: Workload, steps: int, warmup: int, torch, dist, world, flus
             w.geqrf()
             if i is not None:
                 ev[i][1].record(w.stream)
-            if w.nrhs:
+            if w.nrhs and w.kind == "qr":
                 w.apply()
         if i is not None:
             ev[i][2].record(w.stream)
@@ -264,7 +286,9 @@ def roofline_obj(w: Workload, qr_ms: float, peaks: dict, n_sm: int, fused: bool 
                             f"derived: {n_sm} SMs x 128 FP32 lanes x 2 x {peaks.get('sm_max_mhz', 1965.0)} MHz"),
             "roofline_us": round(t_roof * 1e6, 3), "kernel_us": round(qr_ms * 1e3, 3),
             "algorithmic_bytes": nbytes, "useful_flops": flops,
-            "kernel": (w.bqr.load().bqr_qhb_kernel_name(w.code, w.m, w.n, w.nrhs).decode() if fused
+            "kernel": ({"lu": "lu_rf_kernel (LU, no pivoting)", "gj": "lu_rf_kernel (Gauss-Jordan)"}[w.kind]
+                       if w.kind != "qr" else
+                       w.bqr.load().bqr_qhb_kernel_name(w.code, w.m, w.n, w.nrhs).decode() if fused
                        else w.bqr.kernel_name(w.code, w.m, w.n))}
 
 
@@ -319,10 +343,13 @@ def cpu_baseline(name: str, min_seconds: float = 3.0, max_matrices: int | None =
 
 
 def config_block(w: Workload, world, l2_note):
-    return {"workload": f"{w.name}: {w.batch} x {w.m}x{w.n} {w.dt} geqrf" + (f" + Q^H b ({w.nrhs} rhs)" if w.nrhs else "")
-            + " per GPU", "m": w.m, "n": w.n, "batch_per_gpu": w.batch, "global_batch": w.batch * world,
+    op = {"qr": "geqrf" + (f" + Q^H b ({w.nrhs} rhs)" if w.nrhs else ""),
+          "lu": "LU without pivoting (diagonally dominant)",
+          "gj": f"Gauss-Jordan [A | b] ({w.nrhs} rhs, diagonally dominant)"}[w.kind]
+    return {"workload": f"{w.name}: {w.batch} x {w.m}x{w.n} {w.dt} {op} per GPU", "m": w.m, "n": w.n,
+            "batch_per_gpu": w.batch, "global_batch": w.batch * world,
             "dtype": w.dt, "l2": l2_note, "parallelism": f"dp{world} (independent matrices per rank)",
-            "kernel": w.bqr.kernel_name(w.code, w.m, w.n)}
+            "kernel": w.bqr.kernel_name(w.code, w.m, w.n) if w.kind == "qr" else "lu_rf_kernel"}
 
 
 def run_ours(args):
@@ -367,7 +394,7 @@ def run_ours(args):
     out["gpu_launches"] += (e_steps + 2) * 0  # e2e launches are outside the device-timed kernel region
     if not args.no_also:
         also = {}
-        for name in [c for c in ("C4", "C2", "S80", "S192") if c != args.config]:
+        for name in [c for c in ("C4", "C2", "S80", "S192", "L56", "GJ56") if c != args.config]:
             w = Workload(name, rank, world, torch, bqr)
             k2 = max(3, min(args.steps, 100))
             s_ms, q_ms = time_workload(w, k2, max(3, args.warmup), torch, dist, world, flush)
@@ -376,11 +403,11 @@ def run_ours(args):
                           "ms_per_step": round(s_ms, 6), "steps": k2,
                           "matrices_per_s": round(world * w.batch / (s_ms / 1e3), 1),
                           "config": config_block(w, world, l2_note),
-                          "roofline": roofline_obj(w, q_ms, peaks, n_sm, fused=bool(w.nrhs))}
+                          "roofline": roofline_obj(w, q_ms, peaks, n_sm, fused=bool(w.nrhs) and w.kind == "qr")}
             if name in PAPER_TABLE_VII:
                 also[name]["paper_quadro6000_gflops"] = PAPER_TABLE_VII[name]
             out["gpu_launches"] += k2
-            if w.nrhs:
+            if w.nrhs and w.kind == "qr":
                 # context: the same step as two launches (geqrf, then apply_qh)
                 s2, q2 = time_workload(w, k2, max(3, args.warmup), torch, dist, world, flush, fused=False)
                 also[name]["unfused_two_launch"] = {"ms_per_step": round(s2, 6), "geqrf_ms": round(q2, 6),
@@ -441,7 +468,7 @@ def main():
     ap.add_argument("--steps", type=int, default=200)
     ap.add_argument("--warmup", type=int, default=10)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--config", default="C3", choices=["C1", "C2", "C3", "C4", "S80", "S192"])
+    ap.add_argument("--config", default="C3", choices=["C1", "C2", "C3", "C4", "S80", "S192", "L56", "GJ56"])
     ap.add_argument("--no-also", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     args = ap.parse_args()

@@ -35,6 +35,10 @@ CONFIGS = {
     # "80x16 384", "192x96 128"; complex single precision, QR only)
     "S80": dict(m=80, n=16, batch=384, dtype="c64", dist="normal", seed=5),
     "S192": dict(m=192, n=96, batch=128, dtype="c64", dist="normal", seed=6),
+    # NEXT-3: LU without pivoting / Gauss-Jordan, 8,000 problems as the
+    # paper's Fig. 11 comparison, diagonally dominant
+    "L56": dict(m=56, n=56, batch=8000, dtype="f32", dist="diagdom", seed=7, kind="lu"),
+    "GJ56": dict(m=56, n=56, batch=8000, dtype="f32", dist="diagdom", seed=8, nrhs=1, kind="gj"),
 }
 
 
@@ -124,6 +128,8 @@ def config_batch(name: str, start: int = 0, stop: int | None = None,
                  batch: int | None = None) -> np.ndarray:
     cfg = CONFIGS[name]
     b = cfg["batch"] if batch is None else batch
+    if cfg["dist"] == "diagdom":
+        return diag_dominant_batch(cfg["n"], b, cfg["dtype"], cfg["seed"], start=start, stop=stop)
     return random_batch(cfg["m"], cfg["n"], b, cfg["dtype"], cfg["seed"],
                         cfg["dist"], start=start, stop=stop)
 

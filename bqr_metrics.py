@@ -11,6 +11,10 @@ times, pinned in tests/test_metrics.py against the numbers PAPER.md prints.
                           (one reflector application per column, reading Q1)
   algorithmic bytes      read A once, write [R;V] once, write tau;
                           the apply adds B in and out
+  NEXT-3    LU without pivoting "performs 2/3 n^3 FLOPs"
+                          (m x n: m n^2 - n^3/3), Gauss-Jordan "performs n^3
+                          FLOPs"; complex x4.  Bytes: A in and out (+ B in
+                          and out for Gauss-Jordan) + a 4-byte info per matrix.
 """
 from __future__ import annotations
 
@@ -76,3 +80,25 @@ def roofline_time_s(flops: float, nbytes: float, hbm_gbs: float, fp32_tflops: fl
     t_c = flops / (fp32_tflops * 1e12)
     t_m = nbytes / (hbm_gbs * 1e9)
     return (t_c, "alu") if t_c >= t_m else (t_m, "hbm")
+
+
+def lu_flops(m: int, n: int, dtype: str = "f32") -> float:
+    """LU without pivoting, leading order: 2/3 n^3 for square."""
+    k = min(m, n)
+    f = float(m) * n * k - (m + n) * k * k / 2.0 + k ** 3 / 3.0
+    f = 2.0 * f
+    return 4.0 * f if dtype == "c64" else f
+
+
+def gj_flops(n: int, dtype: str = "f32") -> float:
+    """Gauss-Jordan on [A | b]: the paper's n^3."""
+    f = float(n) ** 3
+    return 4.0 * f if dtype == "c64" else f
+
+
+def lu_bytes(m: int, n: int, dtype: str = "f32") -> int:
+    return 2 * m * n * ELEM_BYTES[dtype] + 4
+
+
+def gj_bytes(n: int, nrhs: int, dtype: str = "f32") -> int:
+    return (2 * n * n + 2 * n * nrhs) * ELEM_BYTES[dtype] + 4

@@ -24,6 +24,7 @@ __all__ = [
     "load", "colmajor", "geqrf_batched", "orgqr_batched", "apply_qh_batched",
     "geqrf_batched_host", "host_workspace_bytes", "kernel_name", "geqrf_launches",
     "BQRError", "R32", "C64", "lib_path", "geqrf_batched_ptr", "geqrf_qhb_batched", "gels_batched",
+    "getrf_np_batched", "gauss_jordan_batched",
 ]
 
 R32, C64 = 0, 1
@@ -62,6 +63,11 @@ def load():
     if hasattr(lib, "bqr_gels_batched"):  # absent in older builds (A/B timing)
         lib.bqr_gels_batched.argtypes = [i, i, i, i, i, p, i, p, p, i, p, p]
         lib.bqr_gels_batched.restype = i
+    if hasattr(lib, "bqr_getrf_np_batched"):  # NEXT-3 (absent in older builds)
+        lib.bqr_getrf_np_batched.argtypes = [i, i, i, i, p, i, p, p]
+        lib.bqr_getrf_np_batched.restype = i
+        lib.bqr_gauss_jordan_batched.argtypes = [i, i, i, i, p, i, p, i, p, p]
+        lib.bqr_gauss_jordan_batched.restype = i
     lib.bqr_geqrf_batched_host.argtypes = [i, i, i, i, p, i, p, p, sz, p]
     lib.bqr_host_workspace_bytes.argtypes = [i, i, i, i, i]
     lib.bqr_host_workspace_bytes.restype = sz
@@ -207,6 +213,37 @@ def gels_batched(A, B, tau=None, info=None, stream=None):
                                  ctypes.c_void_p(info.data_ptr()), _stream_ptr(stream))
     _check(st, "bqr_gels_batched")
     return A, tau, B, info
+
+
+def getrf_np_batched(A, info=None, stream=None):
+    """LU without pivoting: A (batch, m, n) column-major per
+    matrix <- L (strict lower) + U.  Returns (A, info) with info (batch,)
+    int32 on the device (0, or k+1 for the first zero pivot)."""
+    import torch
+    batch = A.shape[0]
+    m, n, lda = _layout(A)
+    if info is None:
+        info = torch.empty((batch,), dtype=torch.int32, device=A.device)
+    st = load().bqr_getrf_np_batched(_dtype_code(A), m, n, batch, ctypes.c_void_p(A.data_ptr()), lda,
+                                     ctypes.c_void_p(info.data_ptr()), _stream_ptr(stream))
+    _check(st, "bqr_getrf_np_batched")
+    return A, info
+
+
+def gauss_jordan_batched(A, B, info=None, stream=None):
+    """Gauss-Jordan without pivoting on [A | B]: A (batch, n, n)
+    is destroyed, B (batch, n, nrhs) <- X.  Returns (A, B, info)."""
+    import torch
+    batch = A.shape[0]
+    m, n, lda = _layout(A)
+    _, nrhs, ldb = _layout(B)
+    if info is None:
+        info = torch.empty((batch,), dtype=torch.int32, device=A.device)
+    st = load().bqr_gauss_jordan_batched(_dtype_code(A), n, nrhs, batch, ctypes.c_void_p(A.data_ptr()), lda,
+                                         ctypes.c_void_p(B.data_ptr()), ldb, ctypes.c_void_p(info.data_ptr()),
+                                         _stream_ptr(stream))
+    _check(st, "bqr_gauss_jordan_batched")
+    return A, B, info
 
 
 def host_workspace_bytes(dtype: int, m: int, n: int, lda: int, chunk: int) -> int:

@@ -171,3 +171,41 @@ def test_gels_argument_checks(lib, args, code):
     st = lib.bqr_gels_batched(d, m, n, nrhs, b, ctypes.c_void_p(A), lda, ctypes.c_void_p(tau), ctypes.c_void_p(B),
                               ldb, None, None)
     assert st == code
+
+
+# NEXT-3: LU without pivoting / Gauss-Jordan (argument checks run no kernel)
+@pytest.mark.parametrize("args,code", [
+    ((7, 8, 8, 1, FAKE, 8), -1),
+    ((0, -1, 8, 1, FAKE, 8), -2),
+    ((0, 8, -1, 1, FAKE, 8), -3),
+    ((0, 8, 8, -1, FAKE, 8), -4),
+    ((0, 8, 8, 1, 0, 8), -5),
+    ((0, 8, 8, 1, FAKE, 7), -6),
+    ((0, 8, 8, 0, 0, 8), 0),            # batch == 0: quick return
+    ((0, 0, 8, 5, 0, 1), 0),            # m == 0: quick return
+    ((0, 129, 129, 1, FAKE, 129), 1),   # beyond the size classes
+    ((1, 8, 8, 1, FAKE + 4, 8), 3),     # complex pointer not 8-byte aligned
+])
+def test_getrf_np_argument_checks(lib, args, code):
+    d, m, n, b, A, lda = args
+    st = lib.bqr_getrf_np_batched(d, m, n, b, ctypes.c_void_p(A), lda, None, None)
+    assert st == code
+
+
+@pytest.mark.parametrize("args,code", [
+    ((7, 8, 1, 1, FAKE, 8, FAKE, 8), -1),
+    ((0, -1, 1, 1, FAKE, 8, FAKE, 8), -2),
+    ((0, 8, -1, 1, FAKE, 8, FAKE, 8), -3),
+    ((0, 8, 1, -1, FAKE, 8, FAKE, 8), -4),
+    ((0, 8, 1, 1, 0, 8, FAKE, 8), -5),
+    ((0, 8, 1, 1, FAKE, 7, FAKE, 8), -6),
+    ((0, 8, 1, 1, FAKE, 8, 0, 8), -7),
+    ((0, 8, 1, 1, FAKE, 8, FAKE, 7), -8),
+    ((0, 8, 1, 0, 0, 8, 0, 8), 0),          # batch == 0
+    ((0, 120, 9, 1, FAKE, 120, FAKE, 120), 1),  # n + nrhs > 128
+    ((0, 8, 1, 1, FAKE + 2, 8, FAKE, 8), 3),
+])
+def test_gauss_jordan_argument_checks(lib, args, code):
+    d, n, nrhs, b, A, lda, B, ldb = args
+    st = lib.bqr_gauss_jordan_batched(d, n, nrhs, b, ctypes.c_void_p(A), lda, ctypes.c_void_p(B), ldb, None, None)
+    assert st == code

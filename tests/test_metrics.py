@@ -43,3 +43,15 @@ def test_roofline_bound():
     t, bound = bm.roofline_time_s(1.171e9, 126.6e6, 6545.6, bm.fp32_peak_tflops())
     assert bound == "hbm" and t == pytest.approx(19.34e-6, rel=2e-3)
     assert bm.fp32_peak_tflops() == pytest.approx(74.45, rel=1e-3)
+
+
+def test_next3_flop_counts_match_the_paper():
+    # "This algorithm performs n^3 FLOPs" (Gauss-Jordan);
+    # LU "performs 2/3 n^3 FLOPs"
+    for n in (4, 56, 128):
+        assert bm.gj_flops(n) == n ** 3
+        assert abs(bm.lu_flops(n, n) - 2.0 / 3.0 * n ** 3) < 1e-6 * n ** 3
+    # rectangular LU: m n^2 - n^3/3 (m >= n), symmetric in the wide case
+    assert abs(bm.lu_flops(80, 16) - (80 * 16 ** 2 - 16 ** 3 / 3)) < 1e-9
+    assert abs(bm.lu_flops(16, 80) - bm.lu_flops(80, 16)) < 1e-9
+    assert bm.lu_flops(8, 8, "c64") == 4 * bm.lu_flops(8, 8)
