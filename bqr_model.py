@@ -1,0 +1,162 @@
+"""bqr_model -- NEXT-4: the paper's per-column performance
+model, and the same model re-parameterised for the B200 register-file
+kernels.  Measurement/diagnostics only: no method arithmetic.
+
+The paper (Sec. V-D, Table VI) costs one column of a
+one-problem-per-block QR as
+
+  Column   N g (norm) + (1 + sqrt p) b + sqrt p g (thread-0 reduction)
+           + g_sqrt + 2 g_div + 2 g (scale factor) + 2 b (write/read it)
+           + N g + N b + a_sync (scale the column, write it to shared)
+  Trailing N b (read v) + N^2 g (matvec) + 2 a_sync + (1 + sqrt p) b
+           + sqrt p g (matvec reduction) + N b + N^2 g + a_sync (rank-1)
+
+with N the rows per thread of the live sub-matrix, g the FP pipeline
+latency, b a shared-memory access, a_sync a block barrier (Table IV:
+g = 18, shared latency 27, a_sync = 46 cycles on the Quadro 6000), summed
+over the n - 1 columns; LU per column: g_div + a_sync + 2 b + N g
++ 2 N b + a_sync + 2 N b + N^2 g + a_sync.  ``paper_qr_cycles`` /
+``paper_lu_cycles`` evaluate it (readings: b = the 27-cycle shared latency,
+g_sqrt = g_div = 2 g: the paper took them from a GT200 study it does not
+print); the paper measured 150,203 (QR) and 68,250 (LU) compute cycles for
+56 x 56 (Table V).
+
+On B200 the kernels replace the thread-0 serial reductions by shuffle
+butterflies and overlap the reflector chain with the trailing update
+(look-ahead), so the model has two parts per column k:
+
+  chain_k  the dependent latency from v_k to v_{k+1}: shared-memory read,
+           the slot-P dot (FMA chain), log2 R shuffle+add levels, the
+           update, the norm (FMA chain + log2 R levels + the alpha
+           shuffle), the IEEE sqrt/div chain, the publish (shared write +
+           signal);
+  issue_k  warp instructions a scheduler must issue for its resident
+           groups: 2 Nr Nc FMA instructions per lane (FFMA2 halves them
+           for complex), the reduction shuffles/adds, and a per-step
+           overhead O (masks, loads, scalar chain) calibrated from ncu's
+           executed-instruction count of the bench kernel.
+
+A column then costs between max(chain_k, issue_k) (perfect overlap, IPC 1
+per scheduler) and chain_k + issue_k (no overlap); the kernel takes
+rounds x sum_k of that.  Latencies come from ``tools/micro`` on B200
+(``profiles/micro_r01.jsonl``): FFMA 4.24, shuffle+add 30.2, shared load
+29.0, sqrt.rn + div.rn chain 118 cycles.
+"""
+from __future__ import annotations
+
+import math
+from dataclasses import dataclass
+
+# Table IV, Quadro 6000; readings for the values it does not print
+FERMI = dict(g=18.0, b=27.0, a_sync=46.0, g_sqrt=36.0, g_div=36.0)
+
+# tools/micro on B200 (profiles/micro_r01.jsonl)
+B200 = dict(l_fma=4.24, l_shfl_add=30.17, l_lds=29.02, l_sqrtdiv=118.06, f_ghz=1.965, schedulers=4)
+
+
+def _panels(n_cols: int, width: int):
+    """(columns in panel, panel index) for a 2D-cyclic layout with `width`
+    column groups: panel P holds columns P*width .. P*width+width-1."""
+    P = 0
+    k = 0
+    while k < n_cols:
+        cnt = min(width, n_cols - k)
+        yield cnt, P
+        k += cnt
+        P += 1
+
+
+def paper_qr_cycles(n: int, p: int = 64, prm: dict = FERMI) -> float:
+    """Table VI QR estimate for an n x n matrix on p threads (sqrt p x sqrt p
+    grid), compute only, summed over the n - 1 columns."""
+    g, b, a = prm["g"], prm["b"], prm["a_sync"]
+    sp = int(round(math.sqrt(p)))
+    total = 0.0
+    for cnt, P in _panels(n - 1, sp):
+        N = math.ceil(n / sp) - P  # rows (and columns) per thread in panel P
+        col = N * g + (1 + sp) * b + sp * g + prm["g_sqrt"] + 2 * prm["g_div"] + 2 * g + 2 * b + N * g + N * b + a
+        trail = N * b + N * N * g + 2 * a + (1 + sp) * b + sp * g + N * b + N * N * g + a
+        total += cnt * (col + trail)
+    return total
+
+
+def paper_lu_cycles(n: int, p: int = 64, prm: dict = FERMI) -> float:
+    """Table VI LU estimate (n - 1 columns)."""
+    g, b, a = prm["g"], prm["b"], prm["a_sync"]
+    sp = int(round(math.sqrt(p)))
+    total = 0.0
+    for cnt, P in _panels(n - 1, sp):
+        N = math.ceil(n / sp) - P
+        col = prm["g_div"] + a + 2 * b + N * g + 2 * N * b + a
+        trail = 2 * N * b + N * N * g + a
+        total += cnt * (col + trail)
+    return total
+
+
+@dataclass
+class Layout:
+    """A register-file class: R row lanes x G column groups per matrix,
+    MR x NC elements per lane, `groups_per_warp` matrices per warp (sub-warp
+    groups) or `warps` warps per matrix (CTA groups), `resident` matrices
+    per SM, complex or real, overhead O instructions per lane-step."""
+    m: int
+    n: int
+    R: int
+    G: int
+    MR: int
+    NC: int
+    cplx: bool
+    resident: int           # matrices resident per SM
+    warps_per_matrix: float  # 0.5 = two matrices per warp
+    overhead: float         # per-step instructions besides FMAs and reductions
+    packed: bool = False    # FFMA2 in the matvec / rank-1
+    signal: float = 0.0     # extra cross-warp signal latency per column
+
+
+def column_costs(L: Layout, lat: dict = B200):
+    """Per-column (chain, issue-per-scheduler) cycle estimates."""
+    r = int(round(math.log2(L.R))) if L.R > 1 else 0
+    words = 2 if L.cplx else 1
+    out = []
+    kmax = min(L.m, L.n)
+    for k in range(kmax):
+        P = k // L.G
+        i0 = (P * L.G) // L.R
+        Nr = L.MR - i0
+        Nc = L.NC - P
+        fma_per_mac = (2 if L.packed else 4) if L.cplx else 1
+        chain = (lat["l_lds"] + math.ceil(Nr / 4) * lat["l_fma"] * fma_per_mac + r * lat["l_shfl_add"] * words
+                 + lat["l_fma"] + math.ceil(Nr / 4) * lat["l_fma"] + r * lat["l_shfl_add"] + lat["l_shfl_add"]
+                 + lat["l_sqrtdiv"] * (1.5 if L.cplx else 1.0) + lat["l_lds"] + L.signal)
+        per_lane = 2 * Nr * Nc * fma_per_mac + 2 * r * Nc * words + L.overhead
+        warps_per_sched = L.resident * L.warps_per_matrix / lat["schedulers"]
+        issue = per_lane * warps_per_sched
+        out.append((chain, issue))
+    return out
+
+
+def predict_us(L: Layout, batch: int, n_sm: int = 148, lat: dict = B200) -> dict:
+    """Kernel time bounds (us): rounds x sum over columns of max (overlap)
+    and of the sum (no overlap); the last partial round is costed with the
+    issue of its busiest SM (chain-bound when that is small)."""
+    per_round = batch / (L.resident * n_sm)
+    full = math.floor(per_round)
+    frac = per_round - full
+    cols = column_costs(L, lat)
+    lo_full = sum(max(c, i) for c, i in cols)
+    hi_full = sum(c + i for c, i in cols)
+    # the last round: the busiest SM holds ceil(frac x resident) matrices
+    share = math.ceil(frac * L.resident - 1e-9) / L.resident if frac > 0 else 0.0
+    lo_part = sum(max(c, i * share) for c, i in cols) if frac > 0 else 0.0
+    hi_part = sum(c + i * share for c, i in cols) if frac > 0 else 0.0
+    f = lat["f_ghz"] * 1e3  # cycles per us
+    return {"rounds": per_round, "lo_us": (full * lo_full + lo_part) / f, "hi_us": (full * hi_full + hi_part) / f,
+            "chain_cycles": sum(c for c, _ in cols), "issue_cycles": sum(i for _, i in cols)}
+
+
+# The bench kernels; overhead O calibrated from ncu's
+# executed instructions of the same kernel (profiles/r01/details_*.txt).
+C3_LAYOUT = Layout(m=56, n=56, R=4, G=4, MR=14, NC=14, cplx=False, resident=16, warps_per_matrix=0.5,
+                   overhead=110.0)
+C4_LAYOUT = Layout(m=240, n=66, R=32, G=11, MR=8, NC=6, cplx=True, resident=1, warps_per_matrix=11,
+                   overhead=90.0, packed=True, signal=60.0)
