@@ -655,8 +655,42 @@ struct RfKernel {
     BQR_STAMP(c, k, 1);
     const T ct = X::conj(c.taus[k]);
     const T *vb = c.vbuf + buf(k) * VB + c.rg * MRP;
-    if (!warp_done_slot(c, kk)) apply<P, I0, P, P + 1>(c, a, vb, ct, kk);
     const bool la = kk + 1 < G && k + 1 < c.kmax && warp_has(c, k + 1);
+    if constexpr (Cfg::LAZY) {
+      // CTA groups, one column group per warp (decoupled signalling).
+      // Only the owners of columns k+1 and k+2 need slot P first: the owner
+      // of k+1 forms reflector k+1 from it (look-ahead) and publishes before
+      // anything else; the owner of k+2 applies H_k to slot P only and
+      // defers its other slots to step k+1, after it has published v_{k+2}
+      // (lazy rest-update: otherwise that rest-update sits between v_{k+1}
+      // arriving and the chain of column k+2).  Every other warp applies
+      // H_k to all its live slots in one pass: one reduce-scatter instead
+      // of a separate slot-P butterfly.
+      const bool defer = kk + 2 < G && k + 2 < c.kmax && warp_has(c, k + 2);
+      const bool done = warp_done_slot(c, kk);
+      if (la || defer) {
+        apply<P, I0, P, P + 1>(c, a, vb, ct, kk);
+        if (la) {
+          const Look l = reflector<P, I0>(c, a, k + 1);
+          publish<P, I0>(c, a, k + 1, l, true);
+          sig_arrive(c, k + 1);
+          BQR_STAMP(c, k, 2);
+          if (kk >= 1) {  // the rest-update deferred at step k-1
+            const T ctp = X::conj(c.taus[k - 1]);
+            const T *vbp = c.vbuf + buf(k - 1) * VB + c.rg * MRP;
+            apply<P, I0, P + 1, NC>(c, a, vbp, ctp, kk - 1);
+          }
+          apply<P, I0, P + 1, NC>(c, a, vb, ct, kk);
+        }
+      } else if (done) {
+        apply<P, I0, P + 1, NC>(c, a, vb, ct, kk);
+      } else {
+        apply<P, I0, P, NC>(c, a, vb, ct, kk);
+      }
+      BQR_STAMP(c, k, 3);
+      return;
+    }
+    if (!warp_done_slot(c, kk)) apply<P, I0, P, P + 1>(c, a, vb, ct, kk);
     if constexpr (GT <= 32) {
       // sub-warp groups: the reflector chain (computed unconditionally, no
       // branch around its shuffles) overlaps the remaining updates in one
@@ -666,26 +700,14 @@ struct RfKernel {
       publish<P, I0>(c, a, k + 1, l, la);
       BQR_STAMP(c, k, 3);
     } else {
-      // multi-warp groups: publish first so the other warps never wait.
-      // Lazy rest-update: the warp that will own column k+2 applies H_k only
-      // to its slot P here and defers the other slots to step k+1, after it
-      // has published v_{k+2}; otherwise its whole rest-update of step k
-      // sits between v_{k+1} arriving and the reflector chain of column k+2
-      // (ncu: 15% of warp time in barrier stalls waiting for that chain).
-      const bool defer = Cfg::LAZY && kk + 2 < G && k + 2 < c.kmax && warp_has(c, k + 2);
-      const bool catchup = Cfg::LAZY && la && kk >= 1;
+      // multi-warp groups: publish first so the other warps never wait
       if (la) {
         const Look l = reflector<P, I0>(c, a, k + 1);
         publish<P, I0>(c, a, k + 1, l, true);
         sig_arrive(c, k + 1);
       }
       BQR_STAMP(c, k, 2);
-      if (catchup) {
-        const T ctp = X::conj(c.taus[k - 1]);
-        const T *vbp = c.vbuf + buf(k - 1) * VB + c.rg * MRP;
-        apply<P, I0, P + 1, NC>(c, a, vbp, ctp, kk - 1);
-      }
-      if (!defer) apply<P, I0, P + 1, NC>(c, a, vb, ct, kk);
+      apply<P, I0, P + 1, NC>(c, a, vb, ct, kk);
       BQR_STAMP(c, k, 3);
     }
   }
