@@ -46,6 +46,17 @@ for k in range(nsteps):
     rows.append(dict(k=k, entry_min=int(ent.min()), end_max=int(end.max()),
                      wait=float(np.mean(wt - ent)), slotp=float(np.mean(midv - wt)), rest=float(np.mean(end - midv)),
                      step=int(end.max() - ent.min())))
+# owner analysis (CTA classes with one column group per warp, G = warps):
+# the owner of column k+1 stamps phase 2 right after publishing v_{k+1}
+G = len(warps)
+prev_pub = None
+for k, r in enumerate(rows):
+    w = (k + 1) % G
+    if k + 1 < nsteps and st[k, w, 2] > 0:
+        pub = st[k, w, 2] - t0
+        r["own_chain"] = int(st[k, w, 2] - st[k, w, 1])  # v_k received -> v_{k+1} published
+        r["period"] = int(pub - prev_pub) if prev_pub is not None else None
+        prev_pub = pub
 for r in rows:
     print(json.dumps(r))
 tot = rows[-1]["end_max"] - rows[0]["entry_min"]
