@@ -668,6 +668,7 @@ struct RfKernel {
       // of a separate slot-P butterfly.
       const bool defer = kk + 2 < G && k + 2 < c.kmax && warp_has(c, k + 2);
       const bool done = warp_done_slot(c, kk);
+      int npass;  // rest-updates H_q (slots P+1..), q = k - npass + 1 .. k
       if (la || defer) {
         apply<P, I0, P, P + 1>(c, a, vb, ct, kk);
         if (la) {
@@ -675,18 +676,19 @@ struct RfKernel {
           publish<P, I0>(c, a, k + 1, l, true);
           sig_arrive(c, k + 1);
           BQR_STAMP(c, k, 2);
-          if (kk >= 1) {  // the rest-update deferred at step k-1
-            const T ctp = X::conj(c.taus[k - 1]);
-            const T *vbp = c.vbuf + buf(k - 1) * VB + c.rg * MRP;
-            apply<P, I0, P + 1, NC>(c, a, vbp, ctp, kk - 1);
-          }
-          apply<P, I0, P + 1, NC>(c, a, vb, ct, kk);
         }
+        npass = la ? (kk >= 1 ? 2 : 1) : 0;  // + the rest deferred at step k-1
       } else if (done) {
-        apply<P, I0, P + 1, NC>(c, a, vb, ct, kk);
+        npass = 1;
       } else {
         apply<P, I0, P, NC>(c, a, vb, ct, kk);
+        npass = 0;
       }
+      // one call site for every rest-update (the apply body is inlined per
+      // call site; fewer copies keep the panel code in the instruction cache)
+#pragma unroll 1
+      for (int q = k - npass + 1; q <= k; ++q)
+        apply<P, I0, P + 1, NC>(c, a, c.vbuf + buf(q) * VB + c.rg * MRP, X::conj(c.taus[q]), q - P * G);
       BQR_STAMP(c, k, 3);
       return;
     }
