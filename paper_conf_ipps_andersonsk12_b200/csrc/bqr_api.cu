@@ -204,6 +204,34 @@ size_t elem_size(bqr_dtype_t d) { return d == BQR_R32 ? 4 : 8; }
 
 }  // namespace
 
+// ---- host-buffer pipeline state: two copy streams and the events of a
+// kHostRing-buffer rotation, created once per device (never destroyed;
+// like the kernel attributes) so a call does not pay stream creation
+constexpr int kHostRing = 3;
+struct HostPipe {
+  cudaStream_t h2d = nullptr, d2h = nullptr;
+  cudaEvent_t entry = nullptr, in[kHostRing] = {}, done[kHostRing] = {}, out[kHostRing] = {};
+  bool ok = false;
+};
+
+static HostPipe *host_pipe() {
+  static HostPipe pipes[bqr::host::kMaxDevices];
+  static std::once_flag once[bqr::host::kMaxDevices];
+  const int d = bqr::host::current_device();
+  std::call_once(once[d], [d] {
+    HostPipe &h = pipes[d];
+    bool ok = cudaStreamCreateWithFlags(&h.h2d, cudaStreamNonBlocking) == cudaSuccess &&
+              cudaStreamCreateWithFlags(&h.d2h, cudaStreamNonBlocking) == cudaSuccess &&
+              cudaEventCreateWithFlags(&h.entry, cudaEventDisableTiming) == cudaSuccess;
+    for (int i = 0; i < kHostRing && ok; ++i)
+      ok = cudaEventCreateWithFlags(&h.in[i], cudaEventDisableTiming) == cudaSuccess &&
+           cudaEventCreateWithFlags(&h.done[i], cudaEventDisableTiming) == cudaSuccess &&
+           cudaEventCreateWithFlags(&h.out[i], cudaEventDisableTiming) == cudaSuccess;
+    h.ok = ok;
+  });
+  return pipes[d].ok ? &pipes[d] : nullptr;
+}
+
 extern "C" {
 
 const char *bqr_version(void) { return "bqr 0.1.0 (sm_100a)"; }
@@ -386,12 +414,13 @@ size_t bqr_host_workspace_bytes(bqr_dtype_t dtype, int m, int n, int lda, int ch
   if (!valid_dtype(dtype) || m <= 0 || n <= 0 || chunk <= 0) return 0;
   const size_t s = elem_size(dtype);
   const size_t per = ((size_t)lda * n + std::min(m, n)) * s;
-  return 2 * per * (size_t)chunk + 256;
+  return kHostRing * (per * (size_t)chunk + 512) + 256;
 }
 
-// Host-buffer streaming: chunks of the batch ping-pong through two device
-// buffers; H2D(i+1) overlaps geqrf(i) and D2H(i-1) via two internal streams
-// ordered by events.  Synchronous.
+// Host-buffer streaming: chunks of the batch rotate through kHostRing device
+// buffers; H2D(i+2), geqrf(i+1) and D2H(i) overlap on two internal streams
+// (created once per device, like the kernel attributes) ordered by events.
+// Synchronous.
 int bqr_geqrf_batched_host(bqr_dtype_t dtype, int m, int n, int batch, void *A_host, int lda,
                            void *tau_host, void *workspace, size_t workspace_bytes,
                            cudaStream_t stream) {
@@ -412,65 +441,52 @@ int bqr_geqrf_batched_host(bqr_dtype_t dtype, int m, int n, int batch, void *A_h
   if (m < n) return BQR_ERR_NOT_SUPPORTED;
   Plan p;
   if (!geqrf_plan(dtype, m, n, &p)) return BQR_ERR_NOT_SUPPORTED;
+  constexpr int NB = kHostRing;
   auto r256 = [](size_t x) { return (x + 255) & ~size_t(255); };
-  auto need = [&](long long ch) { return 2 * (r256(mat_bytes * ch) + r256(tau_bytes * ch)) + 256; };
-  long long chunk = std::min<long long>(batch, (long long)(workspace_bytes / (2 * per)));
+  auto need = [&](long long ch) { return NB * (r256(mat_bytes * ch) + r256(tau_bytes * ch)) + 256; };
+  long long chunk = std::min<long long>(batch, (long long)(workspace_bytes / (NB * per)));
   while (chunk > 0 && need(chunk) > workspace_bytes) chunk -= std::max<long long>(1, chunk / 64);
   if (chunk < 1) return -9;
-  // two buffers [A chunk | tau chunk], 256-byte aligned
+  // NB buffers [A chunk | tau chunk], 256-byte aligned
   char *ws = reinterpret_cast<char *>((reinterpret_cast<uintptr_t>(workspace) + 255) & ~uintptr_t(255));
   const size_t abytes = r256(mat_bytes * chunk), tbytes = r256(tau_bytes * chunk);
-  char *bufA[2] = {ws, ws + abytes + tbytes};
-  char *bufT[2] = {ws + abytes, ws + 2 * abytes + tbytes};
-  cudaStream_t st[3] = {stream, nullptr, nullptr};  // compute, h2d, d2h
-  cudaEvent_t ev_in[2], ev_done[2], ev_out[2];
-  int status = BQR_SUCCESS;
-  if (cudaStreamCreateWithFlags(&st[1], cudaStreamNonBlocking) != cudaSuccess ||
-      cudaStreamCreateWithFlags(&st[2], cudaStreamNonBlocking) != cudaSuccess)
-    return BQR_ERR_CUDA;
-  for (int i = 0; i < 2; ++i) {
-    cudaEventCreateWithFlags(&ev_in[i], cudaEventDisableTiming);
-    cudaEventCreateWithFlags(&ev_done[i], cudaEventDisableTiming);
-    cudaEventCreateWithFlags(&ev_out[i], cudaEventDisableTiming);
+  char *bufA[NB], *bufT[NB];
+  for (int i = 0; i < NB; ++i) {
+    bufA[i] = ws + i * (abytes + tbytes);
+    bufT[i] = bufA[i] + abytes;
   }
+  HostPipe *hp = host_pipe();
+  if (!hp) return BQR_ERR_CUDA;
+  cudaStream_t st[3] = {stream, hp->h2d, hp->d2h};  // compute, h2d, d2h
+  int status = BQR_SUCCESS;
   // order the copies after whatever the caller already queued on `stream`
-  cudaEvent_t ev_entry;
-  cudaEventCreateWithFlags(&ev_entry, cudaEventDisableTiming);
-  cudaEventRecord(ev_entry, st[0]);
-  cudaStreamWaitEvent(st[1], ev_entry, 0);
-  cudaEventDestroy(ev_entry);
+  cudaEventRecord(hp->entry, st[0]);
+  cudaStreamWaitEvent(st[1], hp->entry, 0);
   const long long nchunks = (batch + chunk - 1) / chunk;
-  bool out_pending[2] = {false, false};
+  bool out_pending[NB] = {};
   for (long long ci = 0; ci < nchunks && status == BQR_SUCCESS; ++ci) {
-    const int b = (int)(ci & 1);
+    const int b = (int)(ci % NB);
     const long long b0 = ci * chunk;
     const long long cnt = std::min<long long>(chunk, batch - b0);
     // buffer b free once its previous D2H finished
-    if (out_pending[b]) cudaStreamWaitEvent(st[1], ev_out[b], 0);
+    if (out_pending[b]) cudaStreamWaitEvent(st[1], hp->out[b], 0);
     cudaMemcpyAsync(bufA[b], reinterpret_cast<char *>(A_host) + b0 * mat_bytes, cnt * mat_bytes,
                     cudaMemcpyHostToDevice, st[1]);
-    cudaEventRecord(ev_in[b], st[1]);
-    cudaStreamWaitEvent(st[0], ev_in[b], 0);
+    cudaEventRecord(hp->in[b], st[1]);
+    cudaStreamWaitEvent(st[0], hp->in[b], 0);
     Call c{bufA[b], bufT[b], cnt, m, n, k, lda, st[0]};
     status = p.geqrf(c);
-    cudaEventRecord(ev_done[b], st[0]);
-    cudaStreamWaitEvent(st[2], ev_done[b], 0);
+    cudaEventRecord(hp->done[b], st[0]);
+    cudaStreamWaitEvent(st[2], hp->done[b], 0);
     cudaMemcpyAsync(reinterpret_cast<char *>(A_host) + b0 * mat_bytes, bufA[b], cnt * mat_bytes,
                     cudaMemcpyDeviceToHost, st[2]);
     cudaMemcpyAsync(reinterpret_cast<char *>(tau_host) + b0 * tau_bytes, bufT[b], cnt * tau_bytes,
                     cudaMemcpyDeviceToHost, st[2]);
-    cudaEventRecord(ev_out[b], st[2]);
+    cudaEventRecord(hp->out[b], st[2]);
     out_pending[b] = true;
   }
   if (cudaStreamSynchronize(st[2]) != cudaSuccess || cudaStreamSynchronize(st[0]) != cudaSuccess)
     status = BQR_ERR_CUDA;
-  for (int i = 0; i < 2; ++i) {
-    cudaEventDestroy(ev_in[i]);
-    cudaEventDestroy(ev_done[i]);
-    cudaEventDestroy(ev_out[i]);
-  }
-  cudaStreamDestroy(st[1]);
-  cudaStreamDestroy(st[2]);
   if (status == BQR_SUCCESS && cudaGetLastError() != cudaSuccess) status = BQR_ERR_CUDA;
   return status;
 }
