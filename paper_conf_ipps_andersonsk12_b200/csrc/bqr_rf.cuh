@@ -1359,15 +1359,18 @@ struct RfKernel {
 };
 
 // MB = minimum resident CTAs per SM (launch bounds): caps the registers per
-// thread so that MB groups of a small-matrix class share an SM
+// thread so that MB groups of a small-matrix class share an SM.  MB = 1
+// emits no minimum at all: an explicit ".minnctapersm 1" lets ptxas take
+// more registers (e.g. c64 96x96: 198 -> 148 us without it, C3/C4 equal;
+// profiles/r01/experiments/ab_launch_bounds.jsonl)
 template <class T, int R, int G, int MR, int NC, int GPB, bool STAGE, bool EX, bool AUG, int MB = 1>
-__global__ void __launch_bounds__(R * G * GPB, MB) geqrf_rf_kernel(const RfArgs p) {
+__global__ void __launch_bounds__(R * G * GPB, MB > 1 ? MB : 0) geqrf_rf_kernel(const RfArgs p) {
   RfKernel<T, R, G, MR, NC, GPB, STAGE, EX, AUG>::template run<false>(p);
 }
 
 // p.kmax = k (reflectors), p.n = columns of Q, p.tau read-only
 template <class T, int R, int G, int MR, int NC, int GPB, bool STAGE, bool EX, bool AUG, int MB = 1>
-__global__ void __launch_bounds__(R * G * GPB, MB) orgqr_rf_kernel(const RfArgs p) {
+__global__ void __launch_bounds__(R * G * GPB, MB > 1 ? MB : 0) orgqr_rf_kernel(const RfArgs p) {
   RfKernel<T, R, G, MR, NC, GPB, STAGE, EX, AUG>::template run<true>(p);
 }
 
