@@ -530,7 +530,10 @@ struct RfKernel {
       f[2 * j] = wa[j].x + wb[j].y;
       f[2 * j + 1] = wa[j].y - wb[j].x;
     }
-    if constexpr (R >= 8) {
+    // (a single slot -- the owner's slot P on the reflector chain -- takes
+    // plain butterflies: one dependent shuffle stage fewer than the
+    // reduce-scatter + all-gather)
+    if constexpr (R >= 8 && NS >= 2) {
       row_allreduce_multi<R, 2 * NS>(f, c.lane);
     } else {
 #pragma unroll
@@ -601,7 +604,7 @@ struct RfKernel {
         for (int q = 1; q < ACC; ++q) s = X::add(s, w[j][q]);
         sum[j] = s;
       }
-      if constexpr (R >= 8 && NS * Cfg::E >= 2) {
+      if constexpr (R >= 8 && NS * Cfg::E >= 2 && NS >= 2) {
         // several values over >= 8 row lanes: reduce-scatter + all-gather
         float f[NS * Cfg::E];
 #pragma unroll
