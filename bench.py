@@ -300,7 +300,7 @@ def e2e_host(w: Workload, steps: int, warmup: int, torch, dist, world):
     host_in = torch.from_numpy(w.host.copy())
     Ah = torch.empty_like(host_in).pin_memory()
     tauh = torch.empty((w.batch, w.k), dtype=w.tau.dtype).pin_memory()
-    chunk = max(1, w.batch // 8)
+    chunk = max(1, w.batch // 4)  # tools/e2e_ab.py: //4 1.78 ms, //8 1.81, //16 2.06 (B200)
     wsb = bqr.host_workspace_bytes(w.code, w.m, w.n, w.m, chunk)
     ws = torch.empty(wsb, dtype=torch.uint8, device="cuda")
     ev = [[torch.cuda.Event(enable_timing=True) for _ in range(2)] for _ in range(steps)]
