@@ -23,6 +23,15 @@ const ClassEntry kTable[] = {
     {BQR_C64, 240, 72, 0, 0, true, RF_PLAN_AUG(float2, 16, 24, 15, 3, "alt_c64_R16G24_15x3_aug")},
     {BQR_C64, 240, 72, 0, 0, true, RF_PLAN_AUG(float2, 16, 12, 15, 6, "alt_c64_R16G12_15x6_aug")},
     {BQR_C64, 256, 72, 0, 0, true, RF_PLAN_AUG(float2, 32, 24, 8, 3, "alt_c64_R32G24_8x3_aug")},
+    // STAP 80x16 c64 (384 matrices, latency-bound): the former one-warp class and
+    // other thread counts / row-lane splits (experiments/s80_variants.jsonl)
+    {BQR_C64, 80, 16, 80, 16, true, RF_PLAN(float2, 16, 2, 5, 8, 1, false, "alt_c64_R16G2_5x8_warp")},
+    {BQR_C64, 80, 16, 80, 16, true, RF_PLAN(float2, 16, 8, 5, 2, 1, false, "alt_c64_R16G8_5x2_cta")},
+    {BQR_C64, 80, 16, 80, 16, true, RF_PLAN(float2, 8, 4, 10, 4, 1, false, "alt_c64_R8G4_10x4_warp")},
+    {BQR_C64, 96, 16, 0, 0, true, RF_PLAN(float2, 32, 4, 3, 4, 1, false, "alt_c64_R32G4_3x4_cta")},
+    {BQR_C64, 80, 16, 80, 16, true, RF_PLAN(float2, 8, 8, 10, 2, 1, false, "alt_c64_R8G8_10x2_cta")},
+    {BQR_C64, 80, 16, 80, 16, true, RF_PLAN(float2, 16, 16, 5, 1, 1, false, "alt_c64_R16G16_5x1_cta")},
+    {BQR_C64, 80, 16, 80, 16, true, RF_PLAN(float2, 8, 16, 10, 1, 1, false, "alt_c64_R8G16_10x1_cta")},
     // 56x56 fp32, one matrix per warp, register cap for MB warps per SM
     {BQR_R32, 56, 56, 56, 56, true, RF_PLAN_XM(float, 4, 8, 14, 7, 1, true, true, 12, "alt_f32_R4G8_14x7_x1_mb12")},
     {BQR_R32, 56, 56, 56, 56, true, RF_PLAN_XM(float, 4, 8, 14, 7, 1, true, true, 14, "alt_f32_R4G8_14x7_x1_mb14")},

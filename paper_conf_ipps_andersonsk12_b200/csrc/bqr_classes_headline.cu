@@ -12,7 +12,7 @@ const ClassEntry kTable[] = {
     {BQR_R32, 56, 56, 56, 56, false, RF_PLAN_X(float, 4, 4, 14, 14, 2, true, true, "rf_f32_R4G4_14x14_x2_exact")},
     {BQR_C64, 240, 66, 240, 66, false, RF_PLAN(float2, 32, 11, 8, 6, 1, false, "rf_c64_R32G11_8x6_cta")},
     // NEXT-2: the paper's other RT_STAP shapes (Table VII)
-    {BQR_C64, 80, 16, 80, 16, false, RF_PLAN(float2, 16, 2, 5, 8, 1, false, "rf_c64_R16G2_5x8_warp")},
+    {BQR_C64, 80, 16, 80, 16, false, RF_PLAN(float2, 16, 4, 5, 4, 1, false, "rf_c64_R16G4_5x4_cta")},
     {BQR_C64, 192, 96, 192, 96, false, RF_PLAN(float2, 32, 16, 6, 6, 1, false, "rf_c64_R32G16_6x6_cta")},
     {BQR_C64, 256, 72, 240, 67, true, RF_PLAN_AUG(float2, 32, 12, 8, 6, "rf_c64_R32G12_8x6_aug")},
     {BQR_C64, 128, 128, 0, 0, true, RF_PLAN_AUG(float2, 32, 16, 4, 8, "rf_c64_R32G16_4x8_aug")},
