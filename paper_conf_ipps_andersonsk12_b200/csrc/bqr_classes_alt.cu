@@ -32,6 +32,12 @@ const ClassEntry kTable[] = {
     {BQR_C64, 80, 16, 80, 16, true, RF_PLAN(float2, 8, 8, 10, 2, 1, false, "alt_c64_R8G8_10x2_cta")},
     {BQR_C64, 80, 16, 80, 16, true, RF_PLAN(float2, 16, 16, 5, 1, 1, false, "alt_c64_R16G16_5x1_cta")},
     {BQR_C64, 80, 16, 80, 16, true, RF_PLAN(float2, 8, 16, 10, 1, 1, false, "alt_c64_R8G16_10x1_cta")},
+    // STAP 192x96 c64 (128 matrices: one CTA per SM, latency-bound)
+    {BQR_C64, 192, 96, 192, 96, true, RF_PLAN(float2, 32, 32, 6, 3, 1, false, "alt_c64_R32G32_6x3_cta")},
+    {BQR_C64, 192, 96, 192, 96, true, RF_PLAN(float2, 32, 24, 6, 4, 1, false, "alt_c64_R32G24_6x4_cta")},
+    {BQR_C64, 192, 96, 192, 96, true, RF_PLAN(float2, 16, 32, 12, 3, 1, false, "alt_c64_R16G32_12x3_cta")},
+    {BQR_C64, 192, 96, 192, 96, true, RF_PLAN(float2, 16, 16, 12, 6, 1, false, "alt_c64_R16G16_12x6_cta")},
+    {BQR_C64, 192, 96, 192, 96, true, RF_PLAN(float2, 32, 8, 6, 12, 1, false, "alt_c64_R32G8_6x12_cta")},
     // 56x56 fp32, one matrix per warp, register cap for MB warps per SM
     {BQR_R32, 56, 56, 56, 56, true, RF_PLAN_XM(float, 4, 8, 14, 7, 1, true, true, 12, "alt_f32_R4G8_14x7_x1_mb12")},
     {BQR_R32, 56, 56, 56, 56, true, RF_PLAN_XM(float, 4, 8, 14, 7, 1, true, true, 14, "alt_f32_R4G8_14x7_x1_mb14")},
