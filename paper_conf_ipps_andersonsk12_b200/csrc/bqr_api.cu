@@ -61,14 +61,15 @@ using namespace bqr::host;
 // classes, then fp32, then complex64, then the
 // experiment-only alternatives (BQR_FORCE_VARIANT).
 struct Tables {
-  static constexpr int kN = 4;
+  static constexpr int kN = 5;
   const ClassEntry *t[kN];
   int n[kN];
   Tables() {
-    t[0] = classes_headline(&n[0]);
-    t[1] = classes_f32(&n[1]);
-    t[2] = classes_c64(&n[2]);
-    t[3] = classes_alt(&n[3]);
+    t[0] = classes_co(&n[0]);
+    t[1] = classes_headline(&n[1]);
+    t[2] = classes_f32(&n[2]);
+    t[3] = classes_c64(&n[3]);
+    t[4] = classes_alt(&n[4]);
   }
   template <class F>
   const Plan *find(F pred) const {
