@@ -180,3 +180,89 @@ def test_compare_gels_rejects_wrong_solutions():
     conj[:, :, :66] = np.conj(conj[:, :, :66])  # a dropped conjugate
     assert not compare_gels(A_cm, 240, B_cm, conj, info)["ok"]
     assert not compare_gels(A_cm, 240, B_cm, good, info + 1)["ok"]  # wrong info
+
+
+def _householder_sign_rule(A, flip):
+    """Unblocked Householder QR (xGEQR2 form: [R; V], tau) in fp64 with the
+    LAPACK sign rule beta = -copysign(nu, Re alpha) or, flip=True,
+    the opposite sign beta = +copysign(nu, Re alpha) (a self-consistent QR,
+    i.e. A = Q R exactly, that is NOT LAPACK's)."""
+    m, n = A.shape
+    R = A.astype(np.complex128 if np.iscomplexobj(A) else np.float64).copy()
+    taus = []
+    for i in range(min(m, n)):
+        alpha = R[i, i]
+        x = R[i + 1:, i]
+        nu = np.sqrt(abs(alpha) ** 2 + np.vdot(x, x).real)
+        beta = np.copysign(nu, np.real(alpha)) * (1.0 if flip else -1.0)
+        tau = (beta - alpha) / beta
+        v = np.concatenate([[1.0], x / (alpha - beta)])
+        R[i + 1:, i] = v[1:]
+        R[i, i] = beta
+        C = R[i:, i + 1:]
+        C -= np.conj(tau) * np.outer(v, np.conj(v) @ C)
+        taus.append(tau)
+    return R, np.array(taus)
+
+
+@pytest.mark.parametrize("cplx", [False, True])
+def test_rejects_wrong_sign_rule_consistent_qr(cplx):
+    """Every beta sign flipped, V and tau consistent with it: the residual and
+    orthogonality checks pass (it IS a QR of A), so only the comparator's
+    flip rule (oracle margin = |Re alpha|/nu well above 1e-4) can reject it.
+    Pins the margin output of the oracle and the bad-flip rule together: with
+    the margin forced to 0 (every flip 'allowed') this QR would be accepted."""
+    rng = np.random.default_rng(31 + cplx)
+    m, n, batch = 12, 9, 6
+    outs, taus, As = [], [], []
+    for _ in range(batch):
+        A = rng.standard_normal((m, n))
+        if cplx:
+            A = A + 1j * rng.standard_normal((m, n))
+        R, t = _householder_sign_rule(A, flip=True)
+        As.append(A)
+        outs.append(R)
+        taus.append(t)
+    dt = np.complex64 if cplx else np.float32
+    A_cm = oracle.to_cm(np.array(As).astype(dt))
+    out_cm = oracle.to_cm(np.array(outs).astype(dt))
+    rep = compare_geqrf(A_cm, m, out_cm, np.array(taus).astype(dt))
+    assert rep["residual_max"] < 1e-5 and rep["orth_max"] < 1e-5, rep
+    assert rep["bad_flips"] > 0 and not rep["ok"], rep
+    # the rejection comes from the oracle's margins: zeroed, a complex QR
+    # would pass (real ones are also caught by the tau range [1, 2])
+    ref_cm, tau_ref, margin = oracle.geqrf_cm(A_cm, m, with_margin=True)
+    rep0 = compare_geqrf(A_cm, m, out_cm, np.array(taus).astype(dt), ref=(ref_cm, tau_ref, np.zeros_like(margin)))
+    assert rep0["bad_flips"] == 0
+    assert rep0["ok"] if cplx else not rep0["invariants_ok"], rep0
+    # control: the same construction with LAPACK's sign rule is accepted
+    outs = [_householder_sign_rule(A, flip=False) for A in As]
+    rep = compare_geqrf(A_cm, m, oracle.to_cm(np.array([o[0] for o in outs]).astype(dt)),
+                        np.array([o[1] for o in outs]).astype(dt))
+    assert rep["ok"] and rep["bad_flips"] == 0, rep
+
+
+def test_flip_rule_honours_ties():
+    """A flip at an exact tie (margin 0, alpha = +0) is allowed; the same
+    flip where the margin is large is not (bad_flips counts it)."""
+    A = np.array([[0.0, 1.0, 2.0], [1.0, 1.0, 0.5], [0.0, 2.0, 1.0]])
+    _, _, margin = oracle.geqrf(A[None])
+    assert margin[0, 0] == 0.0 and margin[0, 1] > 1e-2
+    R_ok, t_ok = _householder_sign_rule(A, flip=False)
+    # flip only the first reflector (the tie): consistent QR, accepted
+    alpha, x = A[0, 0], A[1:, 0]
+    nu = np.linalg.norm(A[:, 0])
+    beta = +nu
+    tau0 = (beta - alpha) / beta
+    v = np.concatenate([[1.0], x / (alpha - beta)])
+    B = A.copy()
+    B[1:, 0] = v[1:]
+    B[0, 0] = beta
+    C = B[:, 1:]
+    C -= tau0 * np.outer(v, v @ C)
+    Rt, tt = _householder_sign_rule(B[1:, 1:], flip=False)
+    B[1:, 1:] = Rt
+    taus = np.array([tau0, *tt])
+    rep = compare_geqrf(oracle.to_cm(A[None].astype(np.float32)), 3, oracle.to_cm(B[None].astype(np.float32)),
+                        taus[None].astype(np.float32))
+    assert rep["ok"] and rep["flips"] >= 1 and rep["bad_flips"] == 0, rep

@@ -39,9 +39,11 @@ def test_worked_examples(case):
     tau_exp = np.array(case["tau"], dtype=np.float64)
     if cplx:
         tau_exp = tau_exp[..., 0] + 1j * tau_exp[..., 1]
-    RV, tau, _ = oracle.geqrf(A[None])
+    RV, tau, margin = oracle.geqrf(A[None])
     np.testing.assert_allclose(RV[0], RV_exp, rtol=1e-13, atol=1e-14)
     np.testing.assert_allclose(tau[0], tau_exp, rtol=1e-13, atol=1e-14)
+    # the sign-tie margin |alpha|/nu the comparator's flip rule relies on
+    np.testing.assert_allclose(margin[0], np.array(case["margin"]), rtol=1e-13, atol=1e-15)
 
 
 def test_minus_zero_sign_rule():
