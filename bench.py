@@ -2,7 +2,8 @@
 """bench.py -- batched Householder QR on B200: the BASELINE.json metric.
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
-                    [--config C3|C4|C2|C1] [--no-also] [--no-cpu]
+                    [--config C3|C4|C2|C1|...] [--scaling weak|strong]
+                    [--no-also] [--no-c5] [--no-cpu]
 
 One "step" = one pass of the whole hot path over one batch:
   C3 (default, the metric's headline workload): bqr_geqrf_batched on 5,000
@@ -14,8 +15,13 @@ Inputs are seeded synthetic (bqr_inputs) and resident in HBM; before every
 timed step the working buffer is restored from a pristine copy and L2 is
 flushed by writing a 2x-L2 buffer (both untimed); each step is bracketed by
 CUDA events on the launching stream.  Multi-GPU: one process per GPU under
-torchrun, each rank factors its own seeded slice (weak scaling, no data-path
-collective); NCCL only for barriers and the MAX of per-rank times.
+torchrun (`--gpus N` without a torchrun environment re-launches itself under
+torch.distributed.run; a WORLD_SIZE that disagrees with --gpus is an error),
+each rank factors its own seeded slice, no data-path collective; NCCL only
+for barriers and the MAX of per-rank times.  The line's headline is weak
+scaling (per-GPU batch fixed) and it also carries strong scaling (the
+config's batch split over the ranks), the per-matrix latency floor (batch 1,
+one per SM, one resident round) and the C5 size-sweep cells.
 
 --impl reference times the fp64 CPU oracle (oracle/, the parity reference)
 on the host cores on a bounded sample of the same workload.
@@ -119,25 +125,37 @@ def load_traffic(name: str):
 class Workload:
     """Device buffers for one config on one rank."""
 
-    def __init__(self, name, rank, world, torch, bqr, batch=None):
-        cfg = dict(bqr_inputs.CONFIGS[name])
+    def __init__(self, name, rank, world, torch, bqr, batch=None, cfg=None, scaling="weak"):
+        cfg = dict(bqr_inputs.CONFIGS[name] if cfg is None else cfg)
         self.name = name
         self.m, self.n, self.dt = cfg["m"], cfg["n"], cfg["dtype"]
-        self.batch = cfg["batch"] if batch is None else batch
+        total = cfg["batch"] if batch is None else batch
         self.k = min(self.m, self.n)
         self.nrhs = cfg.get("nrhs", 0)
         self.torch, self.bqr = torch, bqr
-        # weak scaling: rank r owns matrices [r*B, (r+1)*B) of a world*B seeded stream
-        lo, hi = bqr_dist.rank_slice(rank, world, self.batch)
         self.kind = cfg.get("kind", "qr")
-        host = bqr_inputs.config_batch(name, start=lo, stop=hi, batch=world * self.batch)
+        if scaling == "weak":
+            # rank r owns matrices [r*B, (r+1)*B) of a world*B seeded stream
+            lo, hi = bqr_dist.rank_slice(rank, world, total)
+            stream_len = world * total
+        else:
+            # strong: the B matrices of the config split floor(r B / P) .. floor((r+1) B / P)
+            lo, hi = bqr_dist.rank_slice(rank, world, 0, weak=False, total=total)
+            stream_len = total
+        self.batch = hi - lo
+        self.global_batch = world * total if scaling == "weak" else total
+        if cfg is not None and name not in bqr_inputs.CONFIGS:
+            host = bqr_inputs.random_batch(self.m, self.n, stream_len, self.dt, cfg["seed"], cfg["dist"],
+                                           start=lo, stop=hi)
+        else:
+            host = bqr_inputs.config_batch(name, start=lo, stop=hi, batch=stream_len)
         self.host = host
         self.pristine = torch.from_numpy(host).cuda()
         self.A = torch.empty_like(self.pristine)
         tdt = self.pristine.dtype
         self.tau = torch.empty((self.batch, self.k), dtype=tdt, device="cuda")
         if self.nrhs:
-            Bh = bqr_inputs.rhs_batch(self.m, self.nrhs, world * self.batch, self.dt, cfg["seed"], start=lo, stop=hi)
+            Bh = bqr_inputs.rhs_batch(self.m, self.nrhs, stream_len, self.dt, cfg["seed"], start=lo, stop=hi)
             self.Bp = torch.from_numpy(Bh).cuda()
             self.B = torch.empty_like(self.Bp)
         self.code = bqr.R32 if self.dt == "f32" else bqr.C64
@@ -163,6 +181,11 @@ class Workload:
             self.bytes_apply = self.batch * bm.apply_bytes(self.m, self.nrhs, self.dt)
         else:
             self.flops_apply = self.bytes_apply = 0
+
+    def step_flops_total(self):
+        """Useful flops of one step over the WHOLE job (all ranks)."""
+        per = (self.flops + self.flops_apply) / max(1, self.batch)
+        return per * self.global_batch
 
     def restore(self):
         self.A.copy_(self.pristine)
@@ -347,9 +370,94 @@ def config_block(w: Workload, world, l2_note):
           "lu": "LU without pivoting (diagonally dominant)",
           "gj": f"Gauss-Jordan [A | b] ({w.nrhs} rhs, diagonally dominant)"}[w.kind]
     return {"workload": f"{w.name}: {w.batch} x {w.m}x{w.n} {w.dt} {op} per GPU", "m": w.m, "n": w.n,
-            "batch_per_gpu": w.batch, "global_batch": w.batch * world,
+            "batch_per_gpu": w.batch, "global_batch": w.global_batch,
             "dtype": w.dt, "l2": l2_note, "parallelism": f"dp{world} (independent matrices per rank)",
             "kernel": w.bqr.kernel_name(w.code, w.m, w.n) if w.kind == "qr" else "lu_rf_kernel"}
+
+
+def latency_scan(w: Workload, torch, dist, world, flush, n_sm: int) -> dict:
+    """Per-matrix latency floor: kernel time of a batch of
+    1 matrix, of one matrix per SM and of one full round of resident matrices
+    (bqr_resident_matrices), L2 flushed, max over ranks."""
+    res = int(w.lib.bqr_resident_matrices(w.code, w.m, w.n))
+    out = {"resident_matrices": res}
+    full = w.batch
+    for label, b in (("batch_1", 1), ("batch_n_sm", n_sm), ("batch_resident", res)):
+        if b <= 0 or b > full:
+            continue
+        w.batch = b
+        _, q_ms = time_workload(w, 20, 3, torch, dist, world, flush)
+        out[f"{label}_us"] = round(q_ms * 1e3, 2)
+    w.batch = full
+    return out
+
+
+C5_CELLS = [(16, "f32"), (56, "f32"), (128, "f32"), (256, "f32"), (16, "c64"), (56, "c64"), (128, "c64"),
+            (256, "c64")]
+
+
+def colnorm_check(w: Workload, torch, stride: int = 97) -> dict:
+    """Property check that holds at any size (Q is unitary): ||R e_j|| equals
+    ||A e_j|| on every `stride`-th matrix plus the first and the last
+    (plain torch on the bench's own output; the oracle parity of the C5 cells
+    at these batch sizes is tests/test_gpu_c5.py)."""
+    w.restore()
+    w.geqrf()
+    torch.cuda.synchronize()
+    idx = sorted(set(range(0, w.batch, stride)) | {w.batch - 1})
+    A = w.pristine[idx].to(torch.complex128 if w.dt == "c64" else torch.float64)  # (s, n, m) storage
+    R = w.A[idx].to(A.dtype)
+    # storage [b, col, row]: upper triangle of the logical matrix = row <= col
+    rows = torch.arange(w.m, device=A.device)[None, None, :]
+    cols = torch.arange(w.n, device=A.device)[None, :, None]
+    Rt = torch.where(rows <= cols, R, torch.zeros_like(R))
+    na = torch.linalg.vector_norm(A, dim=2)
+    nr = torch.linalg.vector_norm(Rt, dim=2)
+    err = float(((nr - na).abs() / na.clamp_min(1e-30)).max())
+    return {"sampled": len(idx), "colnorm_rel_err_max": err, "ok": err < 1e-5}
+
+
+def run_c5(rank, world, torch, dist, bqr, flush, peaks, n_sm, l2_note, steps, warmup):
+    cells = {}
+    launches = 0
+    for n, dt in C5_CELLS:
+        cfg = bqr_inputs.c5_config(n, dt, n_sm=n_sm)
+        name = f"C5_{dt}_{n}"
+        w = Workload(name, rank, world, torch, bqr, cfg=cfg)
+        k2 = max(3, min(steps, 50))
+        s_ms, q_ms = time_workload(w, k2, warmup, torch, dist, world, flush)
+        launches += k2 * int(w.lib.bqr_geqrf_launches(w.code, w.m, w.n, w.batch))
+        cells[name] = {"value": round(w.step_flops_total() / (s_ms / 1e3) / 1e9, 3), "unit": UNIT,
+                       "ms_per_step": round(s_ms, 6), "steps": k2,
+                       "matrices_per_s": round(w.global_batch / (s_ms / 1e3), 1),
+                       "config": config_block(w, world, l2_note),
+                       "roofline": roofline_obj(w, q_ms, peaks, n_sm),
+                       "check": colnorm_check(w, torch)}
+        del w
+        torch.cuda.empty_cache()
+    return cells, launches
+
+
+def dry_run(args, rank, world, torch, dist):
+    """--dry-run: the rank / launch / slicing plumbing of a multi-GPU run
+    without a GPU (gloo): every rank derives its weak and strong slices of
+    the config, they are gathered over the process group, rank 0 prints them
+    (tests/test_dist_gloo.py drives `bench.py --gpus 2 --dry-run`)."""
+    if world > 1:
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        dist.init_process_group("gloo")
+    cfg = bqr_inputs.CONFIGS[args.config]
+    weak = bqr_dist.rank_slice(rank, world, cfg["batch"])
+    strong = bqr_dist.rank_slice(rank, world, 0, weak=False, total=cfg["batch"])
+    t = bqr_dist.max_over_ranks(torch, dist, float(rank))
+    got = bqr_dist.gather_ints(torch, dist, [rank, *weak, *strong])
+    bqr_dist.barrier(torch, dist)
+    if rank == 0:
+        print(json.dumps({"dry_run": True, "n_gpus": world, "config": args.config, "max_rank": t,
+                          "weak_slices": [g[1:3] for g in got], "strong_slices": [g[3:5] for g in got]}),
+              flush=True)
+    if world > 1:
+        dist.destroy_process_group()
 
 
 def run_ours(args):
@@ -357,6 +465,11 @@ def run_ours(args):
     import torch.distributed as dist
     import paper_conf_ipps_andersonsk12_b200 as bqr
     rank, world, local = env_rank()
+    if world != args.gpus:
+        raise SystemExit(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={world} (launch N ranks with torchrun, "
+                         f"or run `python bench.py --gpus N` and let it re-launch itself)")
+    if args.dry_run:
+        return dry_run(args, rank, world, torch, dist)
     torch.cuda.set_device(local)
     if world > 1:
         os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
@@ -369,44 +482,55 @@ def run_ours(args):
     l2_note = f"L2 flushed before every timed step by writing {flush.numel() >> 20} MiB (2x L2); input restored from a pristine copy (untimed)"
     peaks = bm.load_peaks()
 
-    main = Workload(args.config, rank, world, torch, bqr)
+    main = Workload(args.config, rank, world, torch, bqr, scaling=args.scaling)
     sampler = ClockSampler(local)
     step_ms, qr_ms = time_workload(main, args.steps, args.warmup, torch, dist, world, flush, sampler)
-    flops_step = main.flops + main.flops_apply
-    value = world * flops_step / (step_ms / 1e3) / 1e9
+    value = main.step_flops_total() / (step_ms / 1e3) / 1e9
     out = {
         "metric": METRIC, "value": round(value, 3), "unit": UNIT, "n_gpus": world, "steps": args.steps,
-        "warmup": args.warmup, "ms_per_step": round(step_ms, 6), "higher_is_better": True, "scaling": "weak",
+        "warmup": args.warmup, "ms_per_step": round(step_ms, 6), "higher_is_better": True,
+        "scaling": args.scaling,
         "vs_baseline": None, "dtype": "f32" if main.dt == "f32" else "c64", "data": "synthetic (seeded iid Gaussian, bqr_inputs)",
         "config": config_block(main, world, l2_note),
-        "matrices_per_s": round(world * main.batch / (step_ms / 1e3), 1),
+        "matrices_per_s": round(main.global_batch / (step_ms / 1e3), 1),
         "roofline": roofline_obj(main, qr_ms, peaks, n_sm, fused=bool(main.nrhs)),
-        "gpu_launches": args.steps,
+        "gpu_launches": args.steps * int(main.lib.bqr_geqrf_launches(main.code, main.m, main.n, main.batch)),
         "clocks": sampler.summary(),
     }
+    # the other scaling mode at this N (both curves per run)
+    other = "strong" if args.scaling == "weak" else "weak"
+    ow = Workload(args.config, rank, world, torch, bqr, scaling=other)
+    o_ms, o_q = time_workload(ow, max(3, min(args.steps, 100)), args.warmup, torch, dist, world, flush)
+    out[other] = {"value": round(ow.step_flops_total() / (o_ms / 1e3) / 1e9, 3), "unit": UNIT,
+                  "ms_per_step": round(o_ms, 6), "global_batch": ow.global_batch, "batch_per_gpu_max": ow.batch,
+                  "matrices_per_s": round(ow.global_batch / (o_ms / 1e3), 1), "kernel_us": round(o_q * 1e3, 3)}
+    out["gpu_launches"] += max(3, min(args.steps, 100))
+    # per-matrix latency floor (strong-scaling limit)
+    out["latency"] = latency_scan(ow if other == "weak" else main, torch, dist, world, flush, n_sm)
+    del ow
     # end to end through the public host-buffer API
     e_steps = max(3, min(args.steps, 20))
     e_ms, h2d, d2h = e2e_host(main, e_steps, 2, torch, dist, world)
-    out["e2e"] = {"value": round(world * main.flops / (e_ms / 1e3) / 1e9, 3), "unit": UNIT,
-                  "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h, "steps": e_steps,
+    out["e2e"] = {"value": round(main.global_batch * (main.flops / max(1, main.batch)) / (e_ms / 1e3) / 1e9, 3),
+                  "unit": UNIT, "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h, "steps": e_steps,
                   "api": "bqr_geqrf_batched_host (pinned host buffers, chunked H2D/compute/D2H overlap)",
                   "ms_per_step": round(e_ms, 4)}
-    out["gpu_launches"] += (e_steps + 2) * 0  # e2e launches are outside the device-timed kernel region
     if not args.no_also:
         also = {}
         for name in [c for c in ("C4", "C2", "S80", "S192", "L56", "GJ56") if c != args.config]:
-            w = Workload(name, rank, world, torch, bqr)
+            w = Workload(name, rank, world, torch, bqr, scaling=args.scaling)
             k2 = max(3, min(args.steps, 100))
             s_ms, q_ms = time_workload(w, k2, max(3, args.warmup), torch, dist, world, flush)
-            fl = w.flops + w.flops_apply
-            also[name] = {"value": round(world * fl / (s_ms / 1e3) / 1e9, 3), "unit": UNIT,
+            also[name] = {"value": round(w.step_flops_total() / (s_ms / 1e3) / 1e9, 3), "unit": UNIT,
                           "ms_per_step": round(s_ms, 6), "steps": k2,
-                          "matrices_per_s": round(world * w.batch / (s_ms / 1e3), 1),
+                          "matrices_per_s": round(w.global_batch / (s_ms / 1e3), 1),
                           "config": config_block(w, world, l2_note),
                           "roofline": roofline_obj(w, q_ms, peaks, n_sm, fused=bool(w.nrhs) and w.kind == "qr")}
             if name in PAPER_TABLE_VII:
                 also[name]["paper_quadro6000_gflops"] = PAPER_TABLE_VII[name]
             out["gpu_launches"] += k2
+            if name == "C4":
+                also[name]["latency"] = latency_scan(w, torch, dist, world, flush, n_sm)
             if w.nrhs and w.kind == "qr":
                 # context: the same step as two launches (geqrf, then apply_qh)
                 s2, q2 = time_workload(w, k2, max(3, args.warmup), torch, dist, world, flush, fused=False)
@@ -415,6 +539,11 @@ def run_ours(args):
                 out["gpu_launches"] += 2 * k2
             del w
         out["also"] = also
+        if not args.no_c5:
+            cells, nl = run_c5(rank, world, torch, dist, bqr, flush, peaks, n_sm, l2_note, args.steps,
+                               max(3, args.warmup))
+            out["c5"] = cells
+            out["gpu_launches"] += nl
     # determinism evidence (outside the timed region): checksum of one
     # factorised slice per rank, gathered over the process group
     main.restore()
@@ -462,6 +591,20 @@ def run_reference(args):
     print(json.dumps(out), flush=True)
 
 
+def relaunch_under_torchrun(args) -> int:
+    """`python bench.py --gpus N` without a torchrun environment: start N
+    ranks (one process per GPU) on this node through torch.distributed.run,
+    with the same arguments; rank 0 prints the JSON line."""
+    import socket
+    import subprocess
+    with socket.socket() as sk:
+        sk.bind(("127.0.0.1", 0))
+        port = sk.getsockname()[1]
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr=127.0.0.1", f"--master-port={port}", os.path.abspath(__file__), *sys.argv[1:]]
+    return subprocess.call(cmd)
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -469,11 +612,19 @@ def main():
     ap.add_argument("--warmup", type=int, default=10)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--config", default="C3", choices=["C1", "C2", "C3", "C4", "S80", "S192", "L56", "GJ56"])
+    ap.add_argument("--scaling", default="weak", choices=["weak", "strong"],
+                    help="headline mode; the line also carries the other mode at the same N")
     ap.add_argument("--no-also", action="store_true")
+    ap.add_argument("--no-c5", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--dry-run", action="store_true", help="rank/slicing plumbing only (no GPU, gloo)")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3
+    if args.gpus < 1:
+        raise SystemExit("--gpus must be >= 1")
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        sys.exit(relaunch_under_torchrun(args))
     if args.impl == "reference":
         run_reference(args)
     else:

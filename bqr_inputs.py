@@ -124,6 +124,46 @@ def diag_dominant_batch(n: int, batch: int, dtype: str = "f32", seed: int = 0,
     return A
 
 
+STRESS_KINDS = ("tiny", "huge", "graded", "near_rank", "near_rank_tiny")
+
+
+def stress_batch(m: int, n: int, batch: int, dtype: str, kind: str, seed: int) -> np.ndarray:
+    """Inputs at the edges of the stated contract (reading Q6: entries in
+    [1e-15, 1e15] or 0), column-major (batch, n, m):
+      tiny       Gaussian draws with |x| clipped up to 0.1, times 1e-14
+      huge       the same times 1e14
+      graded     column j times 10^(-14 j / (n-1)): columns from O(1) to O(1e-14)
+      near_rank  (B C + 1e-6 E) * 1e-8 with B m x r, C r x n, r = n/2, E noise:
+                 numerical rank r, the trailing columns cancel to ~1e-14
+      near_rank_tiny  the same at 1e-13: the trailing columns cancel to
+                 ~1e-19 and their squares (sigma, nu^2, |z|^2) fall below
+                 FLT_MIN (outside the accuracy contract of reading Q6, which
+                 has no scaled norms; used to check the FTZ guard keeps every
+                 output finite)
+    Only random draws, scaling and a product of random factors (no QR
+    arithmetic)."""
+    A = random_batch(m, n, batch, dtype, seed).astype(np.complex128 if dtype == "c64" else np.float64)
+    if kind in ("tiny", "huge", "graded"):
+        mag = np.maximum(np.abs(A), 0.1)
+        A = np.where(np.abs(A) > 0, A / np.where(np.abs(A) > 0, np.abs(A), 1.0), 1.0) * mag
+        if kind == "tiny":
+            A = A * 1e-14
+        elif kind == "huge":
+            A = A * 1e14
+        else:
+            A = A * (10.0 ** (-14.0 * np.arange(n) / max(1, n - 1)))[None, :, None]
+    elif kind in ("near_rank", "near_rank_tiny"):
+        r = max(1, n // 2)
+        Bf = random_batch(m, r, batch, dtype, seed + 1).astype(A.dtype)   # (batch, r, m): B^T storage
+        Cf = random_batch(r, n, batch, dtype, seed + 2).astype(A.dtype)   # (batch, n, r)
+        # storage [b, col, row]: (B C)[row, col] = sum_t B[row, t] C[t, col]
+        BC = np.einsum("btr,bct->bcr", Bf, Cf)
+        A = (BC + 1e-6 * A) * (1e-13 if kind == "near_rank_tiny" else 1e-8)
+    else:
+        raise ValueError(kind)
+    return A.astype(np_dtype(dtype))
+
+
 def config_batch(name: str, start: int = 0, stop: int | None = None,
                  batch: int | None = None) -> np.ndarray:
     cfg = CONFIGS[name]

@@ -77,6 +77,14 @@ def load():
     lib.bqr_status_string.restype = ctypes.c_char_p
     lib.bqr_kernel_name.argtypes = [i, i, i]
     lib.bqr_kernel_name.restype = ctypes.c_char_p
+    if hasattr(lib, "bqr_resident_matrices"):  # (older builds, e.g. A/B libraries, lack the diagnostics)
+        lib.bqr_resident_matrices.argtypes = [i, i, i]
+        lib.bqr_resident_matrices.restype = ctypes.c_longlong
+        lib.bqr_class_count.argtypes = []
+        lib.bqr_class_count.restype = i
+        ip = ctypes.POINTER(ctypes.c_int)
+        lib.bqr_class_info.argtypes = [i, ip, ip, ip, ip, ip, ip]
+        lib.bqr_class_info.restype = ctypes.c_char_p
     lib.bqr_geqrf_launches.argtypes = [i, i, i, i]
     lib.bqr_geqrf_launches.restype = i
     lib.bqr_version.restype = ctypes.c_char_p
@@ -257,6 +265,22 @@ def geqrf_batched_host(dtype: int, m: int, n: int, batch: int, A_host_ptr: int, 
                                        ctypes.c_void_p(tau_host_ptr), ctypes.c_void_p(workspace_ptr),
                                        workspace_bytes, _stream_ptr(stream))
     _check(st, "bqr_geqrf_batched_host")
+
+
+def size_classes() -> list:
+    """The library's size-class table (bqr_class_info): one dict per entry
+    with dtype, mmax, nmax, exact_m, exact_n, experiment, augmented,
+    dispatched (picked by bqr_geqrf_batched) and name."""
+    lib = load()
+    out = []
+    vals = [ctypes.c_int() for _ in range(6)]
+    for idx in range(lib.bqr_class_count()):
+        name = lib.bqr_class_info(idx, *[ctypes.byref(v) for v in vals])
+        dt, mmax, nmax, em, en, fl = (v.value for v in vals)
+        out.append({"name": name.decode(), "dtype": dt, "mmax": mmax, "nmax": nmax, "exact_m": em,
+                    "exact_n": en, "experiment": bool(fl & 1), "augmented": bool(fl & 2),
+                    "dispatched": not (fl & 4)})
+    return out
 
 
 def kernel_name(dtype: int, m: int, n: int) -> str:

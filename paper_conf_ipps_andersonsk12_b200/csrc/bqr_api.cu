@@ -148,8 +148,10 @@ int apply_dispatch_t(bqr_dtype_t dt, const ApplyArgs &a, cudaStream_t s) {
 // to the trailing columns by the Q^H B kernel, on panel views of the batch
 // (custom batch strides; 2 launches per panel).
 bool tiled_panel_width(bqr_dtype_t dt, int m, int n, int *nb) {
-  if (m > 256) return false;
-  *nb = dt == BQR_R32 ? 64 : 96;  // widest tall class: fp32 256x64, c64 256x96
+  // fp32 up to 256 x 256 always has a single-SM class (bqr_classes_f32.cu),
+  // so only complex shapes beyond 160 x 160 take the tiled path
+  if (m > 256 || dt != BQR_C64) return false;
+  *nb = 96;  // widest tall complex class: 256 x 96
   return n > *nb;
 }
 
@@ -210,6 +212,7 @@ size_t elem_size(bqr_dtype_t d) { return d == BQR_R32 ? 4 : 8; }
 // like the kernel attributes) so a call does not pay stream creation
 constexpr int kHostRing = 3;
 struct HostPipe {
+  std::mutex mu;  // one host call at a time per device: the events and copy streams are shared
   cudaStream_t h2d = nullptr, d2h = nullptr;
   cudaEvent_t entry = nullptr, in[kHostRing] = {}, done[kHostRing] = {}, out[kHostRing] = {};
   bool ok = false;
@@ -261,10 +264,44 @@ const char *bqr_kernel_name(bqr_dtype_t dtype, int m, int n) {
   Plan p;
   if (!geqrf_plan(dtype, m, n, &p)) {
     int nb;
-    return tiled_panel_width(dtype, m, n, &nb) ? (dtype == BQR_R32 ? "tiled_f32_panel64+apply" : "tiled_c64_panel96+apply")
-                                                : "";
+    return tiled_panel_width(dtype, m, n, &nb) ? "tiled_c64_panel96+apply" : "";
   }
   return p.name ? p.name : "";
+}
+
+long long bqr_resident_matrices(bqr_dtype_t dtype, int m, int n) {
+  if (!valid_dtype(dtype) || m <= 0 || n <= 0 || m < n) return 0;
+  Plan p;
+  if (!geqrf_plan(dtype, m, n, &p)) return 0;  // tiled oversize path: several launches
+  long long r = 0;
+  Call c{nullptr, nullptr, 1, m, n, std::min(m, n), m, nullptr};
+  c.resident = &r;
+  return p.geqrf(c) == BQR_SUCCESS ? r : 0;
+}
+
+int bqr_class_count(void) {
+  int total = 0;
+  tables().each([&](const ClassEntry &) { ++total; });
+  return total;
+}
+
+const char *bqr_class_info(int index, int *dtype, int *mmax, int *nmax, int *exact_m, int *exact_n, int *flags) {
+  if (index < 0) return nullptr;
+  const ClassEntry *found = nullptr;
+  int i = 0;
+  tables().each([&](const ClassEntry &e) {
+    if (i++ == index) found = &e;
+  });
+  if (!found) return nullptr;
+  if (dtype) *dtype = found->dt;
+  if (mmax) *mmax = found->mmax;
+  if (nmax) *nmax = found->nmax;
+  if (exact_m) *exact_m = found->exact_m;
+  if (exact_n) *exact_n = found->exact_n;
+  const bool aug = std::strstr(found->plan.name, "_aug") != nullptr;
+  const bool experiment = std::strncmp(found->plan.name, "alt_", 4) == 0;
+  if (flags) *flags = (experiment ? 1 : 0) | (aug ? 2 : 0) | (found->alt ? 4 : 0);
+  return found->plan.name;
 }
 
 int bqr_geqrf_launches(bqr_dtype_t dtype, int m, int n, int batch) {
@@ -380,6 +417,7 @@ int bqr_orgqr_batched(bqr_dtype_t dtype, int m, int n, int k, int batch, void *A
   Plan p;
   if (!orgqr_plan(dtype, m, n, &p)) return BQR_ERR_NOT_SUPPORTED;
   Call c{A, const_cast<void *>(tau), batch, m, n, k, lda, stream};
+  c.strideT = n;  // tau batch stride min(m, n) = n, as bqr_geqrf_batched wrote it
   return p.orgqr(c);
 }
 
@@ -401,7 +439,9 @@ int bqr_apply_qh_batched(bqr_dtype_t dtype, int m, int n, int k, int nrhs, int b
   if ((reinterpret_cast<uintptr_t>(A) | reinterpret_cast<uintptr_t>(tau) |
        reinterpret_cast<uintptr_t>(B)) % elem_size(dtype))
     return BQR_ERR_MISALIGNED;
-  ApplyArgs a{A, tau, B, batch, lda, n, m, k, nrhs, ldb, (long long)lda * n, (long long)k, (long long)ldb * nrhs};
+  // tau batch stride min(m, n): the stride bqr_geqrf_batched wrote, also when k < min(m, n)
+  ApplyArgs a{A, tau, B, batch, lda, n, m, k, nrhs, ldb, (long long)lda * n, (long long)std::min(m, n),
+              (long long)ldb * nrhs};
   return apply_dispatch_t(dtype, a, stream);
 }
 
@@ -458,6 +498,11 @@ int bqr_geqrf_batched_host(bqr_dtype_t dtype, int m, int n, int batch, void *A_h
   }
   HostPipe *hp = host_pipe();
   if (!hp) return BQR_ERR_CUDA;
+  // re-entrancy: concurrent host calls on one device are serialised (the
+  // call is synchronous anyway); without the lock thread B could re-record
+  // done[b] between thread A's record and wait, and A's D2H would copy back
+  // before its own kernel ran
+  std::lock_guard<std::mutex> lock(hp->mu);
   cudaStream_t st[3] = {stream, hp->h2d, hp->d2h};  // compute, h2d, d2h
   int status = BQR_SUCCESS;
   // order the copies after whatever the caller already queued on `stream`

@@ -16,6 +16,10 @@ int launch_co(const Call &c) {
   if (!ok) return FB(c);
   auto kern = geqrf_co_kernel<M, N, L, H, LS, PW, MINB>;
   if (!ensure_smem(reinterpret_cast<const void *>(kern), Cf::SMEM)) return BQR_ERR_CUDA;
+  if (c.resident) {
+    *c.resident = resident_of(reinterpret_cast<const void *>(kern), 128, Cf::SMEM, Cf::WPC * Cf::MPW);
+    return BQR_SUCCESS;
+  }
   const long long items = (c.batch + Cf::MPW - 1) / Cf::MPW;
   long long grid = (items + Cf::WPC - 1) / Cf::WPC;
   int sms = 0, bps = 0;

@@ -41,7 +41,18 @@ struct Call {
   void *B = nullptr;  // fused Q^H B (augmented columns); direct-load classes only
   int ldb = 1, nrhs = 0;
   long long strideA = -1, strideT = -1;  // batch strides; -1 = LAPACK-contiguous
+  // non-null: report how many matrices of this shape are resident on the
+  // current device at once (occupancy x matrices per CTA) and launch nothing
+  long long *resident = nullptr;
 };
+
+// occupancy-based residency of a kernel: CTAs per SM x SMs x matrices per CTA
+inline long long resident_of(const void *kern, int threads, size_t smem, long long per_cta) {
+  int sms = 0, bps = 0;
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, current_device());
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, kern, threads, smem);
+  return (long long)sms * bps * per_cta;
+}
 
 using LaunchFn = int (*)(const Call &);
 
@@ -92,6 +103,10 @@ int launch_rf(const Call &c) {
                       (prefetch ? mat_bytes : 0);
   auto kern = ORG ? orgqr_rf_kernel<T, R, G, MR, NC, GPB, STAGE, EX, AUG, MB> : geqrf_rf_kernel<T, R, G, MR, NC, GPB, STAGE, EX, AUG, MB>;
   if (!ensure_smem(reinterpret_cast<const void *>(kern), smem)) return BQR_ERR_CUDA;
+  if (c.resident) {
+    *c.resident = resident_of(reinterpret_cast<const void *>(kern), Cfg::NT, smem, GPB);
+    return BQR_SUCCESS;
+  }
   long long grid = (c.batch + GPB - 1) / GPB;
   // sub-warp exact-shape kernels run a persistent prefetching warp loop when
   // the batch is contiguous (a.bulk)
@@ -119,6 +134,10 @@ int launch_tiny(const Call &c) {
   a.lda = c.lda;
   a.staged = (K::kCanStage && c.lda == M && (reinterpret_cast<uintptr_t>(c.A) & 15) == 0) ? 1 : 0;
   const long long per_block = 32LL * K::kWarps;
+  if (c.resident) {
+    *c.resident = resident_of(reinterpret_cast<const void *>(geqrf_tiny_kernel<T, M, N>), K::kWarps * 32, 0, per_block);
+    return BQR_SUCCESS;
+  }
   const long long grid = (c.batch + per_block - 1) / per_block;
   if (grid > 0x7fffffffLL) return BQR_ERR_NOT_SUPPORTED;
   geqrf_tiny_kernel<T, M, N><<<(unsigned)grid, K::kWarps * 32, 0, c.stream>>>(a);

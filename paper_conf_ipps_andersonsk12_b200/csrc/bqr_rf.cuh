@@ -233,6 +233,20 @@ struct RfKernel {
   // ~250 KB of straight-line code thrashes the instruction cache (58% of
   // stall samples "no_inst" on B200), so the panel loop is the default.
   static constexpr bool kFullUnroll = false;
+  // 1: one butterfly per column on the owner's chain (apply_look) and the
+  // cross-panel look-ahead; correct (parity green) but slower on every
+  // measured class (C3 92 -> 140 us, C4 118 -> 130 us: three reflector
+  // copies per panel body, profiles/r02/experiments/README.md), so the
+  // default is the round-1 chain (dot butterfly, then the norm butterfly)
+#ifndef BQR_FUSED_LOOK
+#define BQR_FUSED_LOOK 0
+#endif
+  static constexpr bool kFusedLook = BQR_FUSED_LOOK != 0;
+  // the last step of a panel forms the next panel's first reflector
+#ifndef BQR_CROSS_PANEL
+#define BQR_CROSS_PANEL 1
+#endif
+  static constexpr bool kCross = BQR_CROSS_PANEL != 0 && kFusedLook;
   static __device__ __forceinline__ int buf(int k) { return k % NBUF; }
 
   struct Ctx {
@@ -348,6 +362,98 @@ struct RfKernel {
     return l;
   }
 
+  // Look-ahead slot P fused with the reflector of column kn = k+1 (the
+  // owner's chain of one step, Table VI "Column" after "Trailing Matrix"):
+  // H_k is unitary on rows >= k, so the squared norm of the updated column
+  // over rows >= k equals gamma = sum_{r >= k} |a_r|^2 of the column BEFORE
+  // the update, and nu^2 = |alpha|^2 + sigma = gamma - |a'_k|^2 with a'_k =
+  // R_{k,kn} and alpha = a'_kn read from the two updated pivot rows.  gamma
+  // rides in the same butterfly as the dot product w = v^H a, so the chain
+  // has one row reduction per column instead of two.  The subtraction is
+  // accurate while it cancels at most one bit (nu^2 >= gamma / 2); below
+  // that, or when sigma may be (near) zero (|alpha|^2 > 15/16 nu^2, e.g. an
+  // already triangular column, which must give tau = 0 exactly, reading Q5),
+  // the group falls back to the direct masked norm of reflector() -- a
+  // warp-uniform branch, rare on dense inputs.
+  // S: the slot holding column kn (P, or P + 1 for the cross-panel
+  // look-ahead of a panel's last step); rows from I0; register rows
+  // [IM, IM + NM) may hold rows k / kn; I0F: first register row of kn's panel
+  // (the fallback reflector and its masks).
+  template <int S, int I0, int IM, int NM, int I0F>
+  static __device__ __forceinline__ Look apply_look(Ctx &c, T (&a)[MR][NC], const T *vb, T ct, int k, bool la) {
+    const int kn = k + 1;
+    T v[MR];
+    load_v<I0>(vb, v);
+    T w0 = X::zero(), w1 = X::zero();
+    float g0 = 0.f, g1 = 0.f;
+    const int limk = k - c.rg;  // row r = rg + R i >= k  <=>  R i >= limk
+#pragma unroll
+    for (int i = I0; i < MR; ++i) {
+      const T x = a[i][S];
+      if ((i - I0) & 1) {
+        w1 = X::cfma(v[i], x, w1);
+      } else {
+        w0 = X::cfma(v[i], x, w0);
+      }
+      const T xm = (i >= IM && i < IM + NM) ? X::sel(R * i >= limk, x, X::zero()) : (i < IM ? X::zero() : x);
+      if ((i - I0) & 1) {
+        g1 = X::abs2_acc(xm, g1);
+      } else {
+        g0 = X::abs2_acc(xm, g0);
+      }
+    }
+    T w = X::add(w0, w1);
+    float gam = g0 + g1;
+    if constexpr (R > 1) {
+      if constexpr (X::kComplex) {
+        float f[3] = {X::re(w), X::im(w), gam};
+#pragma unroll
+        for (int o = 1; o < R; o <<= 1) {
+#pragma unroll
+          for (int q = 0; q < 3; ++q) f[q] += __shfl_xor_sync(0xffffffffu, f[q], o);
+        }
+        w = X::make(f[0], f[1]);
+        gam = f[2];
+      } else {
+        float f[2] = {X::re(w), gam};
+#pragma unroll
+        for (int o = 1; o < R; o <<= 1) {
+#pragma unroll
+          for (int q = 0; q < 2; ++q) f[q] += __shfl_xor_sync(0xffffffffu, f[q], o);
+        }
+        w = X::make(f[0], 0.f);
+        gam = f[1];
+      }
+    }
+    const T t = X::sel(S * G + c.cg > k, X::mul(ct, w), X::zero());
+#pragma unroll
+    for (int i = I0; i < MR; ++i) a[i][S] = X::fnms(v[i], t, a[i][S]);
+    // the updated pivot rows k and kn of this column
+    T xk = X::zero(), xa = X::zero();
+    const int limn = kn - c.rg;
+#pragma unroll
+    for (int i = IM; i < MR && i < IM + NM; ++i) {
+      xk = X::sel(R * i == limk, a[i][S], xk);
+      xa = X::sel(R * i == limn, a[i][S], xa);
+    }
+    if constexpr (R > 1) {
+      xk = X::shfl(xk, (c.lane & ~(R - 1)) | (k & (R - 1)));
+      xa = X::shfl(xa, (c.lane & ~(R - 1)) | (kn & (R - 1)));
+    }
+    const float xk2 = X::abs2_acc(xk, 0.f), xa2 = X::abs2_acc(xa, 0.f);
+    const float nu2 = gam - xk2;
+    const float sig = nu2 - xa2;
+    const bool own = la && ((GT > 32 && R == 32) ? true : (c.cg == kn % G));
+    const bool bad = own && !(nu2 >= 0.5f * gam && sig >= 0.0625f * nu2);
+    if (__any_sync(0xffffffffu, bad)) return reflector<S, I0F>(c, a, kn);
+    const Reflector<T> h = make_reflector(xa, sig);
+    Look l;
+    l.scal = h.scal;
+    l.tau = h.tau;
+    l.beta = h.beta;
+    return l;
+  }
+
   // Owner lanes (own && on): scale the column, store beta, publish v and
   // tau.  Branch-free, so no divergent region precedes the next shuffles
   // (a divergent branch makes the compiler guard every later shuffle with
@@ -431,7 +537,8 @@ struct RfKernel {
   // is the same fma as the scalar path; only the summation grouping of the
   // dot products differs (two interleaved partial sums per accumulator).
   template <int P, int I0, int J0, int J1>
-  static __device__ __forceinline__ void apply_pk_real(Ctx &c, float (&a)[MR][NC], const float *vb, float ct, int kk) {
+  static __device__ __forceinline__ void apply_pk_real(Ctx &c, float (&a)[MR][NC], const float *vb, float ct, int kk,
+                                                     bool skip0 = false) {
     constexpr int NS = J1 - J0;
     constexpr int IP = (I0 + 1) & ~1;
     constexpr int NPR = (MR - IP) / 2;
@@ -481,6 +588,7 @@ struct RfKernel {
     for (int j = 0; j < NS; ++j) {
       tw[j] = ct * sum[j];
       if (J0 + j == P) tw[j] = c.cg > kk ? tw[j] : 0.f;
+      if (j == 0) tw[j] = skip0 ? 0.f : tw[j];
     }
     {
       float v[MR];
@@ -506,7 +614,7 @@ struct RfKernel {
   // a = fma2((vr, vr), (-tr, -ti), a); a = fma2((vi, vi), (ti, -tr), a).
   template <int P, int I0, int J0, int J1>
   static __device__ __forceinline__ void apply_pk_cplx(Ctx &c, float2 (&a)[MR][NC], const float2 *vb, float2 ct,
-                                                      int kk) {
+                                                      int kk, bool skip0 = false) {
     constexpr int NS = J1 - J0;
     float2 wa[NS], wb[NS];
 #pragma unroll
@@ -544,6 +652,7 @@ struct RfKernel {
     for (int j = 0; j < NS; ++j) {
       float2 t = X::mul(ct, pk(f[2 * j], f[2 * j + 1]));
       if (J0 + j == P) t = X::sel(c.cg > kk, t, X::zero());
+      if (j == 0) t = X::sel(skip0, X::zero(), t);
       n1[j] = pk(-t.x, -t.y);
       n2[j] = pk(t.y, -t.x);
     }
@@ -560,11 +669,11 @@ struct RfKernel {
   }
 
   template <int P, int I0, int J0, int J1>
-  static __device__ __forceinline__ void apply_pk(Ctx &c, T (&a)[MR][NC], const T *vb, T ct, int kk) {
+  static __device__ __forceinline__ void apply_pk(Ctx &c, T (&a)[MR][NC], const T *vb, T ct, int kk, bool skip0) {
     if constexpr (X::kComplex)
-      apply_pk_cplx<P, I0, J0, J1>(c, a, vb, ct, kk);
+      apply_pk_cplx<P, I0, J0, J1>(c, a, vb, ct, kk, skip0);
     else
-      apply_pk_real<P, I0, J0, J1>(c, a, vb, ct, kk);
+      apply_pk_real<P, I0, J0, J1>(c, a, vb, ct, kk, skip0);
   }
 
   // ------------------------------------------------------------ trailing update
@@ -572,9 +681,11 @@ struct RfKernel {
   // columns with cg <= kk are excluded (already factored).  The vector is
   // re-read from shared memory in 16-byte chunks for each pass.
   template <int P, int I0, int J0, int J1>
-  static __device__ __forceinline__ void apply(Ctx &c, T (&a)[MR][NC], const T *vb, T ct, int kk) {
+  // skip0: leave slot J0 alone (the cross-panel look-ahead already applied
+  // H_k to it); a uniform select on its multiplier
+  static __device__ __forceinline__ void apply(Ctx &c, T (&a)[MR][NC], const T *vb, T ct, int kk, bool skip0 = false) {
     if constexpr (kPacked && J0 < J1) {
-      apply_pk<P, I0, J0, J1>(c, a, vb, ct, kk);
+      apply_pk<P, I0, J0, J1>(c, a, vb, ct, kk, skip0);
     } else if constexpr (J0 < J1) {
       constexpr int NS = J1 - J0;
       // partial sums per slot: ptxas walks the slots one after another, so a
@@ -624,6 +735,7 @@ struct RfKernel {
       for (int j = 0; j < NS; ++j) {
         tw[j] = X::mul(ct, sum[j]);
         if (J0 + j == P) tw[j] = X::sel(c.cg > kk, tw[j], X::zero());
+        if (j == 0) tw[j] = X::sel(skip0, X::zero(), tw[j]);
       }
       {
         T v[MR];
@@ -649,7 +761,35 @@ struct RfKernel {
 
   // one Householder step on column k of panel P (first live register row I0):
   // apply H_k to slot P, form + publish reflector k+1 (same slot), then apply
-  // H_k to the remaining slots while the reflector chain drains.
+  // H_k to the remaining slots while the reflector chain drains.  The last
+  // step of a panel (kCross) runs the look-ahead on slot P + 1 instead --
+  // column k+1 opens the next panel -- so no panel starts with a reflector
+  // that nothing overlaps (panel_head runs for panel 0 only).
+  template <int P, int I0>
+  static __device__ __forceinline__ Look look(Ctx &c, T (&a)[MR][NC], const T *vb, T ct, int k, bool la) {
+    if constexpr (kFusedLook) {
+      return apply_look<P, I0, I0, Cfg::NMASK, I0>(c, a, vb, ct, k, la);
+    } else {
+      apply<P, I0, P, P + 1>(c, a, vb, ct, k - P * G);
+      return reflector<P, I0>(c, a, k + 1);
+    }
+  }
+  // look-ahead across the panel boundary: H_k on slot P + 1 and reflector
+  // k+1 = (P+1) G from it (rows from I0; the pivot rows k, k+1 lie in
+  // register rows [I0, I0 + NMASK + 1); the next panel starts at row I0N)
+  template <int P, int I0>
+  static __device__ __forceinline__ Look look_x(Ctx &c, T (&a)[MR][NC], const T *vb, T ct, int k, bool la) {
+    constexpr int PN = P + 1 < NC ? P + 1 : P;
+    constexpr int I0N = (PN * G) / R;
+    return apply_look<PN, I0, I0, Cfg::NMASK + 1, I0N>(c, a, vb, ct, k, la);
+  }
+  template <int P>
+  static __device__ __forceinline__ void publish_x(Ctx &c, T (&a)[MR][NC], int kn, const Look &l, bool on) {
+    constexpr int PN = P + 1 < NC ? P + 1 : P;
+    constexpr int I0N = (PN * G) / R;
+    publish<PN, I0N>(c, a, kn, l, on);
+  }
+
   template <int P, int I0>
   static __device__ __forceinline__ void step(Ctx &c, T (&a)[MR][NC], int k) {
     const int kk = k - P * G;
@@ -659,6 +799,9 @@ struct RfKernel {
     const T ct = X::conj(c.taus[k]);
     const T *vb = c.vbuf + buf(k) * VB + c.rg * MRP;
     const bool la = kk + 1 < G && k + 1 < c.kmax && warp_has(c, k + 1);
+    // cross-panel look-ahead (last step of the panel, a next panel exists)
+    const bool lastx = kCross && (P + 1 < NC) && kk == G - 1 && k + 1 < c.kmax;
+    const bool lax = lastx && warp_has(c, k + 1);
     if constexpr (Cfg::LAZY) {
       // CTA groups, one column group per warp (decoupled signalling).
       // Only the owners of columns k+1 and k+2 need slot P first: the owner
@@ -672,15 +815,23 @@ struct RfKernel {
       const bool defer = kk + 2 < G && k + 2 < c.kmax && warp_has(c, k + 2);
       const bool done = warp_done_slot(c, kk);
       int npass;  // rest-updates H_q (slots P+1..), q = k - npass + 1 .. k
+      bool skip = false;
       if (la || defer) {
-        apply<P, I0, P, P + 1>(c, a, vb, ct, kk);
         if (la) {
-          const Look l = reflector<P, I0>(c, a, k + 1);
+          const Look l = look<P, I0>(c, a, vb, ct, k, true);
           publish<P, I0>(c, a, k + 1, l, true);
           sig_arrive(c, k + 1);
           BQR_STAMP(c, k, 2);
+        } else {
+          apply<P, I0, P, P + 1>(c, a, vb, ct, kk);
         }
         npass = la ? (kk >= 1 ? 2 : 1) : 0;  // + the rest deferred at step k-1
+      } else if (lax) {
+        const Look l = look_x<P, I0>(c, a, vb, ct, k, true);
+        publish_x<P>(c, a, k + 1, l, true);
+        sig_arrive(c, k + 1);
+        npass = 1;
+        skip = true;
       } else if (done) {
         npass = 1;
       } else {
@@ -691,28 +842,48 @@ struct RfKernel {
       // call site; fewer copies keep the panel code in the instruction cache)
 #pragma unroll 1
       for (int q = k - npass + 1; q <= k; ++q)
-        apply<P, I0, P + 1, NC>(c, a, c.vbuf + buf(q) * VB + c.rg * MRP, X::conj(c.taus[q]), q - P * G);
+        apply<P, I0, P + 1, NC>(c, a, c.vbuf + buf(q) * VB + c.rg * MRP, X::conj(c.taus[q]), q - P * G,
+                                skip && q == k);
       BQR_STAMP(c, k, 3);
       return;
     }
-    if (!warp_done_slot(c, kk)) apply<P, I0, P, P + 1>(c, a, vb, ct, kk);
     if constexpr (GT <= 32) {
       // sub-warp groups: the reflector chain (computed unconditionally, no
       // branch around its shuffles) overlaps the remaining updates in one
       // basic block; the owner lanes publish at the end of the step
-      const Look l = reflector<P, I0>(c, a, k + 1);
-      apply<P, I0, P + 1, NC>(c, a, vb, ct, kk);
-      publish<P, I0>(c, a, k + 1, l, la);
+      // (one call site of the rest-update; the second test of lastx is
+      // opaque so the compiler does not thread the branch through it by
+      // duplicating the update)
+      Look l;
+      if (lastx) {
+        l = look_x<P, I0>(c, a, vb, ct, k, true);
+      } else {
+        l = look<P, I0>(c, a, vb, ct, k, la);
+      }
+      apply<P, I0, P + 1, NC>(c, a, vb, ct, kk, lastx);
+      if (opaque(lastx ? 1 : 0)) {
+        publish_x<P>(c, a, k + 1, l, true);
+      } else {
+        publish<P, I0>(c, a, k + 1, l, la);
+      }
       BQR_STAMP(c, k, 3);
     } else {
       // multi-warp groups: publish first so the other warps never wait
+      bool skip = false;
       if (la) {
-        const Look l = reflector<P, I0>(c, a, k + 1);
+        const Look l = look<P, I0>(c, a, vb, ct, k, true);
         publish<P, I0>(c, a, k + 1, l, true);
         sig_arrive(c, k + 1);
+      } else if (lax) {
+        const Look l = look_x<P, I0>(c, a, vb, ct, k, true);
+        publish_x<P>(c, a, k + 1, l, true);
+        sig_arrive(c, k + 1);
+        skip = true;
+      } else if (!warp_done_slot(c, kk)) {
+        apply<P, I0, P, P + 1>(c, a, vb, ct, kk);
       }
       BQR_STAMP(c, k, 2);
-      apply<P, I0, P + 1, NC>(c, a, vb, ct, kk);
+      apply<P, I0, P + 1, NC>(c, a, vb, ct, kk, skip);
       BQR_STAMP(c, k, 3);
     }
   }
@@ -881,7 +1052,7 @@ struct RfKernel {
         return;
       }
       const int kend = min(kbeg + G, c.kmax);
-      panel_head<P, I0>(c, a, kbeg);
+      if (P == 0 || !kCross) panel_head<P, I0>(c, a, kbeg);
 #pragma unroll 1
       for (int k = kbeg; k < kend; ++k) step<P, I0>(c, a, k);
       panels<P + 1>(c, a, hook);
@@ -1278,6 +1449,10 @@ struct RfKernel {
             a[i][j] = x;
           }
       } else {
+        // last matrix of this warp: the previous iteration's bulk store may
+        // still be reading the tile when no prefetch hook drained it
+        if (t == 0) bulk_store_drain();
+        warp_sync();
 #pragma unroll
         for (int i = 0; i < MR; ++i)
 #pragma unroll

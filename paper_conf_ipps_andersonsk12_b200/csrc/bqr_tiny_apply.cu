@@ -36,7 +36,8 @@ Plan tiny_plan(int m, int n) {
 
 // self-test of the branch-free IEEE helpers (bqr_common.cuh) against the
 // CUDA library's sqrt.rn / div.rn on random normal operands spanning the
-// exponent range the contract (reading Q6) can produce.
+// exponent range the contract (reading Q6) can produce, plus subnormal
+// operands (the FTZ guard).
 __device__ __forceinline__ unsigned hash32(unsigned x) {
   x ^= x >> 16; x *= 0x7feb352dU; x ^= x >> 15; x *= 0x846ca68bU; x ^= x >> 16;
   return x;
@@ -47,7 +48,7 @@ __device__ __forceinline__ float rand_normal_float(unsigned h, int emin, int ema
   return __uint_as_float(((unsigned)(e + 127) << 23) | mant);
 }
 __global__ void selftest_math_kernel(long long n, unsigned seed, unsigned long long *counts) {
-  unsigned long long bad_sqrt = 0, bad_div = 0, bad_rcp = 0;
+  unsigned long long bad_sqrt = 0, bad_div = 0, bad_rcp = 0, bad_sub = 0;
   for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x) {
     const unsigned h1 = hash32((unsigned)i * 2654435761U ^ seed), h2 = hash32(h1 ^ 0x9e3779b9U);
     const float x = rand_normal_float(h1, -100, 100);           // sigma / |z|^2 range
@@ -56,10 +57,14 @@ __global__ void selftest_math_kernel(long long n, unsigned seed, unsigned long l
     bad_sqrt += __float_as_uint(bqr::sqrt_rn(x)) != __float_as_uint(__fsqrt_rn(x));
     bad_div += __float_as_uint(bqr::div_rn(a, b)) != __float_as_uint(__fdiv_rn(a, b));
     bad_rcp += __float_as_uint(bqr::div_rn(1.0f, b)) != __float_as_uint(__frcp_rn(b));
+    // subnormal operands of the square root (the FTZ guard)
+    const float xs = __uint_as_float((h1 & 0x7fffffU) | 1u);  // nonzero (sqrt_rn(0) is the caller's skip case)
+    bad_sub += __float_as_uint(bqr::sqrt_rn(xs)) != __float_as_uint(__fsqrt_rn(xs));
   }
   atomicAdd(&counts[0], bad_sqrt);
   atomicAdd(&counts[1], bad_div);
   atomicAdd(&counts[2], bad_rcp);
+  atomicAdd(&counts[3], bad_sub);
 }
 
 template <class T>

@@ -74,3 +74,39 @@ def test_generator_slices_independent_of_chunking():
     full = bqr_inputs.random_batch(4, 4, 300, "c64", seed=3, chunk=64)
     part = bqr_inputs.random_batch(4, 4, 300, "c64", seed=3, start=100, stop=231, chunk=64)
     np.testing.assert_array_equal(full[100:231], part)
+
+
+def _bench_env():
+    env = {k: v for k, v in os.environ.items() if k not in ("RANK", "WORLD_SIZE", "LOCAL_RANK", "MASTER_PORT")}
+    env["CUDA_VISIBLE_DEVICES"] = ""
+    return env
+
+
+def test_bench_relaunches_itself_under_torchrun():
+    """`python bench.py --gpus 2` (no torchrun environment) starts 2 ranks via
+    torch.distributed.run; the ranks agree on the weak and strong slices of
+    the C3 batch and rank 0 prints one JSON line (gloo, CPU)."""
+    import json
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    r = subprocess.run([sys.executable, os.path.join(root, "bench.py"), "--gpus", "2", "--dry-run"],
+                       capture_output=True, text=True, timeout=240, env=_bench_env(), cwd=root)
+    assert r.returncode == 0, r.stderr[-3000:]
+    lines = [ln for ln in r.stdout.splitlines() if ln.startswith("{")]
+    assert len(lines) == 1, r.stdout
+    out = json.loads(lines[0])
+    assert out["n_gpus"] == 2 and out["max_rank"] == 1.0
+    assert out["weak_slices"] == [[0, 5000], [5000, 10000]]
+    assert out["strong_slices"] == [[0, 2500], [2500, 5000]]
+
+
+def test_bench_rejects_world_size_mismatch():
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    env = _bench_env()
+    env.update(WORLD_SIZE="2", RANK="0", LOCAL_RANK="0")
+    r = subprocess.run([sys.executable, os.path.join(root, "bench.py"), "--gpus", "4", "--dry-run"],
+                       capture_output=True, text=True, timeout=120, env=env, cwd=root)
+    assert r.returncode != 0 and "WORLD_SIZE=2" in r.stderr

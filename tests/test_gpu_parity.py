@@ -221,6 +221,40 @@ def test_host_buffer_api():
     assert np.array_equal(tau_h.numpy().view(np.uint32), dev_tau.view(np.uint32))
 
 
+def test_host_buffer_api_two_threads():
+    """Re-entrancy of bqr_geqrf_batched_host (include/bqr.h): two host threads
+    on one device, each with its own stream, host buffers and workspace, run
+    many chunked calls concurrently; every result equals the device path bit
+    for bit (ctypes releases the GIL during the call)."""
+    import threading
+
+    import paper_conf_ipps_andersonsk12_b200 as bqr
+    jobs = []
+    for t in range(2):
+        A = bqr_inputs.random_batch(56, 56, 600, "f32", seed=90 + t)
+        ref_out, ref_tau = geqrf_gpu(A, 56)
+        wsb = bqr.host_workspace_bytes(bqr.R32, 56, 56, 56, 64)
+        jobs.append(dict(A=A, ref=(ref_out, ref_tau), ws=torch.empty(wsb, dtype=torch.uint8, device="cuda"),
+                         wsb=wsb, stream=torch.cuda.Stream(), ok=[]))
+    torch.cuda.synchronize()
+
+    def work(j):
+        for _ in range(6):
+            Ah = torch.from_numpy(j["A"].copy()).pin_memory()
+            tau_h = torch.empty((600, 56), dtype=torch.float32).pin_memory()
+            bqr.geqrf_batched_host(bqr.R32, 56, 56, 600, Ah.data_ptr(), 56, tau_h.data_ptr(), j["ws"].data_ptr(),
+                                   j["wsb"], stream=j["stream"])
+            j["ok"].append(np.array_equal(Ah.numpy().view(np.uint32), j["ref"][0].view(np.uint32))
+                           and np.array_equal(tau_h.numpy().view(np.uint32), j["ref"][1].view(np.uint32)))
+
+    th = [threading.Thread(target=work, args=(j,)) for j in jobs]
+    for t in th:
+        t.start()
+    for t in th:
+        t.join()
+    assert all(len(j["ok"]) == 6 and all(j["ok"]) for j in jobs), [j["ok"] for j in jobs]
+
+
 @pytest.mark.parametrize("dt,m,n,nrhs", [("c64", 240, 66, 1), ("c64", 240, 66, 4), ("c64", 80, 16, 2),
                                          ("f32", 100, 30, 3), ("f32", 56, 56, 1), ("c64", 8, 8, 1)])
 def test_fused_geqrf_qhb(dt, m, n, nrhs):
