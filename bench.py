@@ -427,12 +427,13 @@ def run_c5(rank, world, torch, dist, bqr, flush, peaks, n_sm, l2_note, steps, wa
         k2 = max(3, min(steps, 50))
         s_ms, q_ms = time_workload(w, k2, warmup, torch, dist, world, flush)
         launches += k2 * int(w.lib.bqr_geqrf_launches(w.code, w.m, w.n, w.batch))
-        cells[name] = {"value": round(w.step_flops_total() / (s_ms / 1e3) / 1e9, 3), "unit": UNIT,
-                       "ms_per_step": round(s_ms, 6), "steps": k2,
-                       "matrices_per_s": round(w.global_batch / (s_ms / 1e3), 1),
-                       "config": config_block(w, world, l2_note),
-                       "roofline": roofline_obj(w, q_ms, peaks, n_sm),
-                       "check": colnorm_check(w, torch)}
+        cell = {"value": round(w.step_flops_total() / (s_ms / 1e3) / 1e9, 3), "unit": UNIT,
+                "ms_per_step": round(s_ms, 6), "steps": k2,
+                "matrices_per_s": round(w.global_batch / (s_ms / 1e3), 1),
+                "config": config_block(w, world, l2_note),
+                "roofline": roofline_obj(w, q_ms, peaks, n_sm),
+                "check": colnorm_check(w, torch)}
+        cells[name] = cell
         del w
         torch.cuda.empty_cache()
     return cells, launches

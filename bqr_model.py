@@ -160,3 +160,55 @@ C3_LAYOUT = Layout(m=56, n=56, R=4, G=4, MR=14, NC=14, cplx=False, resident=16, 
                    overhead=110.0)
 C4_LAYOUT = Layout(m=240, n=66, R=32, G=11, MR=8, NC=6, cplx=True, resident=1, warps_per_matrix=11,
                    overhead=90.0, packed=True, signal=60.0)
+
+
+# ----------------------------------------------------------------------------
+# Round 2: bounds that price the issue stalls (NEXT-4).
+#
+# Microbenchmarks on B200 (tools/micro/micro2.cu -> profiles/r02/micro2.jsonl,
+# in-kernel clock64 cycles): FFMA latency 4.43, shuffle + add 30.3, shared
+# load 29.0, IEEE sqrt + div chain 118, mbarrier hand-off between two warps
+# 98, named barrier (64 threads) 29, __syncthreads 16 (32 thr) .. 77 (1024),
+# cluster barrier 355-379, DSMEM remote load 202-226; FP32 pipe at 8-16
+# resident warps: FFMA 92, FFMA2 83-88 FMA / clk / SM (of 128); shared
+# memory 127.5 B / clk / SM (Table II analogue).
+B200_R2 = dict(l_fma=4.43, l_shfl_add=30.33, l_lds=29.02, l_sqrtdiv=122.0, l_mbar=98.0, f_ghz=1.965,
+               schedulers=4, fma_per_clk_sm=92.0)
+
+
+def bounds_us(L: Layout, batch: int, instr_total: float, cpi_warp: float, useful_fmas: float,
+              n_sm: int = 148, lat: dict = B200_R2) -> dict:
+    """Lower / upper bounds of one launch from measured counts.
+
+    lo = the largest of three lower bounds: issue (every warp instruction of
+         the launch, ncu ``inst_executed``, at 1 per scheduler per cycle),
+         FP32 pipe (useful FMAs at the measured FFMA rate) and the reflector
+         chain (rounds x sum of the per-column dependent latency, which no
+         schedule can shorten);
+    hi = ceil(rounds) x (the chain fully exposed + the instructions of one
+         warp per round x the measured warp CPI, ncu "warp cycles per issued
+         instruction", i.e. the issue stalls of this kernel at its
+         occupancy): every round paid at full contention, the last (partial)
+         one included, nothing of the chain hidden.
+    The per-matrix latency floor (batch 1, the strong-scaling limit) is the
+    chain plus one warp's instructions at CPI 1 (lo1) ... at the measured
+    CPI (hi1)."""
+    f = lat["f_ghz"] * 1e3
+    slots = L.resident * n_sm
+    rounds = batch / slots
+    warps = max(1.0, batch * L.warps_per_matrix)             # warp-iterations of the launch
+    per_warp_round = instr_total / warps                     # instructions of one warp per matrix group
+    cols = column_costs(L, {**B200, **{k: v for k, v in lat.items() if k in B200}})
+    chain = sum(c for c, _ in cols)
+    issue = instr_total / (lat["schedulers"] * n_sm)
+    fma = useful_fmas / (lat["fma_per_clk_sm"] * n_sm)
+    lo = max(issue, fma, math.ceil(rounds - 1e-9) * chain)
+    hi = math.ceil(rounds - 1e-9) * (chain + per_warp_round * cpi_warp)
+    return {"rounds": rounds, "lo_us": lo / f, "hi_us": hi / f,
+            "lo_terms_us": {"issue": issue / f, "fp32_pipe": fma / f, "chain": math.ceil(rounds - 1e-9) * chain / f},
+            "chain_cycles_per_matrix": chain, "instr_per_warp_round": per_warp_round, "cpi_warp": cpi_warp,
+            "latency_floor_us": {"lo": (chain + per_warp_round) / f, "hi": (chain + per_warp_round * cpi_warp) / f}}
+
+
+S80_LAYOUT = Layout(m=80, n=16, R=16, G=4, MR=5, NC=4, cplx=True, resident=8, warps_per_matrix=2,
+                    overhead=60.0, packed=True, signal=29.0)

@@ -77,6 +77,13 @@ def load():
     lib.bqr_status_string.restype = ctypes.c_char_p
     lib.bqr_kernel_name.argtypes = [i, i, i]
     lib.bqr_kernel_name.restype = ctypes.c_char_p
+    if hasattr(lib, "bqr_geqrf_wy_batched"):  # compact-WY blocked variant (absent in older builds)
+        lib.bqr_geqrf_wy_batched.argtypes = [i, i, i, i, p, i, p, p, sz, p]
+        lib.bqr_geqrf_wy_batched.restype = i
+        lib.bqr_geqrf_wy_workspace_bytes.argtypes = [i, i, i, i, i]
+        lib.bqr_geqrf_wy_workspace_bytes.restype = sz
+        lib.bqr_geqrf_wy_kernel_name.argtypes = [i, i, i, i]
+        lib.bqr_geqrf_wy_kernel_name.restype = ctypes.c_char_p
     if hasattr(lib, "bqr_resident_matrices"):  # (older builds, e.g. A/B libraries, lack the diagnostics)
         lib.bqr_resident_matrices.argtypes = [i, i, i]
         lib.bqr_resident_matrices.restype = ctypes.c_longlong
@@ -265,6 +272,18 @@ def geqrf_batched_host(dtype: int, m: int, n: int, batch: int, A_host_ptr: int, 
                                        ctypes.c_void_p(tau_host_ptr), ctypes.c_void_p(workspace_ptr),
                                        workspace_bytes, _stream_ptr(stream))
     _check(st, "bqr_geqrf_batched_host")
+
+
+def geqrf_wy_workspace_bytes(dtype: int, m: int, n: int, lda: int, chunk: int) -> int:
+    return int(load().bqr_geqrf_wy_workspace_bytes(dtype, m, n, lda, chunk))
+
+
+def geqrf_wy_batched_ptr(dtype: int, m: int, n: int, batch: int, A_ptr: int, lda: int, tau_ptr: int,
+                         work_ptr: int, work_bytes: int, stream=None) -> int:
+    """Compact-WY blocked QR (tensor-core trailing updates) through the C ABI;
+    returns the status code."""
+    return load().bqr_geqrf_wy_batched(dtype, m, n, batch, ctypes.c_void_p(A_ptr), lda, ctypes.c_void_p(tau_ptr),
+                                       ctypes.c_void_p(work_ptr), work_bytes, _stream_ptr(stream))
 
 
 def size_classes() -> list:

@@ -18,6 +18,19 @@ FLAGS = [
 ]
 
 
+def cutlass_flags():
+    """CUTLASS / CuTe headers vendored in the image (flashinfer's copy): used
+    by bqr_wy.cu's tensor-core GEMMs; without them that translation unit
+    compiles to stubs (the blocked WY entry point then falls back)."""
+    import site
+    for sp in site.getsitepackages():
+        inc = os.path.join(sp, "flashinfer", "data", "cutlass", "include")
+        if os.path.isdir(os.path.join(inc, "cutlass")):
+            util = os.path.join(sp, "flashinfer", "data", "cutlass", "tools", "util", "include")
+            return ["-I" + inc, "-I" + util, "--expt-relaxed-constexpr", "-diag-suppress", "20012"]
+    return ["-DBQR_NO_CUTLASS"]
+
+
 def sources():
     out = []
     for d, _, files in os.walk(CSRC):
@@ -44,7 +57,8 @@ def build(force: bool = False, verbose: bool = False, extra=()) -> str:
     procs = []
     for u in units:
         obj = os.path.join(objdir, u[:-3] + ".o")
-        cmd = [NVCC, *cflags, *extra, "-c", "-o", obj, os.path.join(CSRC, u)]
+        cmd = [NVCC, *cflags, *(cutlass_flags() if u == "bqr_wy.cu" else []), *extra, "-c", "-o", obj,
+               os.path.join(CSRC, u)]
         if verbose:
             cmd.insert(1, "-Xptxas=-v")
             print(" ".join(cmd), file=sys.stderr)
@@ -55,7 +69,7 @@ def build(force: bool = False, verbose: bool = False, extra=()) -> str:
             raise subprocess.CalledProcessError(pr.returncode, f"nvcc {u}")
         objs.append(obj)
     link = [NVCC, "-shared", "-gencode", "arch=compute_100a,code=sm_100a", "-Xcompiler", "-fPIC",
-            "-o", LIB + ".tmp", *objs]
+            "-o", LIB + ".tmp", *objs, "-lcuda"]
     subprocess.check_call(link)
     os.replace(LIB + ".tmp", LIB)
     return LIB

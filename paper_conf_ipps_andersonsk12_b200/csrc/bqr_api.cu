@@ -155,6 +155,60 @@ bool tiled_panel_width(bqr_dtype_t dt, int m, int n, int *nb) {
   return n > *nb;
 }
 
+// compact-WY blocked variant (bqr_wy.cu) for the complex shapes beyond one
+// SM: 96-column register panels + tensor-core trailing updates
+const Plan *pick_c64_panel(int m, int n) { return pick(BQR_C64, m, n); }
+constexpr int kWyPanel = 96;
+constexpr size_t kWyMaxWorkspace = size_t(2) << 30;  // stream-ordered workspace cap of the default path
+
+bool wy_default(bqr_dtype_t dt, int m, int n, int lda, const void *A) {
+  return wy_supported(dt, m, n, lda) && (reinterpret_cast<uintptr_t>(A) & 15) == 0;
+}
+
+// a library-private stream-ordered memory pool per device that keeps its
+// memory between calls (release threshold: unlimited), so repeated calls do
+// not remap the workspace; created once, like the kernel attributes
+cudaMemPool_t wy_pool() {
+  static cudaMemPool_t pools[kMaxDevices] = {};
+  static std::once_flag once[kMaxDevices];
+  const int d = current_device();
+  std::call_once(once[d], [d] {
+    cudaMemPoolProps props = {};
+    props.allocType = cudaMemAllocationTypePinned;
+    props.location.type = cudaMemLocationTypeDevice;
+    props.location.id = d;
+    cudaMemPool_t p = nullptr;
+    if (cudaMemPoolCreate(&p, &props) == cudaSuccess) {
+      unsigned long long thr = ~0ULL;
+      cudaMemPoolSetAttribute(p, cudaMemPoolAttrReleaseThreshold, &thr);
+      pools[d] = p;
+    } else {
+      cudaGetLastError();
+    }
+  });
+  return pools[d];
+}
+
+// bqr_geqrf_batched's path for those shapes: the blocked variant on a
+// workspace taken from the library's stream-ordered memory pool on the
+// caller's stream (cudaMallocFromPoolAsync / cudaFreeAsync: no host
+// synchronisation, private to this call); the tiled path if the pool cannot
+// provide it
+int geqrf_wy_default(int m, int n, long long batch, void *A, int lda, void *tau, cudaStream_t stream) {
+  const size_t per = wy_workspace_bytes(m, n, 1, kWyPanel);
+  const long long chunk = std::max<long long>(1, std::min<long long>(batch, (long long)(kWyMaxWorkspace / per)));
+  const size_t bytes = wy_workspace_bytes(m, n, (int)chunk, kWyPanel);
+  cudaMemPool_t pool = wy_pool();
+  void *ws = nullptr;
+  if (!pool || cudaMallocFromPoolAsync(&ws, bytes, pool, stream) != cudaSuccess) {
+    cudaGetLastError();
+    return BQR_ERR_NOT_SUPPORTED;
+  }
+  const int st = geqrf_wy(m, n, batch, A, lda, tau, ws, bytes, kWyPanel, stream, &pick_c64_panel);
+  cudaFreeAsync(ws, stream);
+  return st;
+}
+
 int geqrf_tiled(bqr_dtype_t dt, int m, int n, long long batch, void *A, int lda, void *tau, int nb,
                 cudaStream_t stream) {
   const int kmax = std::min(m, n);
@@ -264,7 +318,9 @@ const char *bqr_kernel_name(bqr_dtype_t dtype, int m, int n) {
   Plan p;
   if (!geqrf_plan(dtype, m, n, &p)) {
     int nb;
-    return tiled_panel_width(dtype, m, n, &nb) ? "tiled_c64_panel96+apply" : "";
+    if (!tiled_panel_width(dtype, m, n, &nb)) return "";
+    return (wy_supported(dtype, m, n, m) && !forced_variant()) ? "wy_c64_panel96+tcgen05_fastf32_gemm"
+                                                              : "tiled_c64_panel96+apply";
   }
   return p.name ? p.name : "";
 }
@@ -277,6 +333,38 @@ long long bqr_resident_matrices(bqr_dtype_t dtype, int m, int n) {
   Call c{nullptr, nullptr, 1, m, n, std::min(m, n), m, nullptr};
   c.resident = &r;
   return p.geqrf(c) == BQR_SUCCESS ? r : 0;
+}
+
+// ---- compact-WY blocked variant (bqr_wy.cu): explicit workspace entry point
+
+size_t bqr_geqrf_wy_workspace_bytes(bqr_dtype_t dtype, int m, int n, int lda, int chunk) {
+  if (!valid_dtype(dtype) || m <= 0 || n <= 0 || chunk <= 0) return 0;
+  if (!wy_supported(dtype, m, n, lda)) return 0;
+  return wy_workspace_bytes(m, n, chunk, kWyPanel);
+}
+
+const char *bqr_geqrf_wy_kernel_name(bqr_dtype_t dtype, int m, int n, int lda) {
+  if (!valid_dtype(dtype) || m <= 0 || n <= 0 || m < n) return "";
+  if (!wy_supported(dtype, m, n, lda)) return bqr_kernel_name(dtype, m, n);
+  return "wy_c64_panel96+tcgen05_fastf32_gemm";
+}
+
+int bqr_geqrf_wy_batched(bqr_dtype_t dtype, int m, int n, int batch, void *A, int lda, void *tau, void *work,
+                         size_t work_bytes, cudaStream_t stream) {
+  if (!valid_dtype(dtype)) return -1;
+  if (m < 0) return -2;
+  if (n < 0) return -3;
+  if (batch < 0) return -4;
+  const bool work_needed = m > 0 && n > 0 && batch > 0;
+  if (work_needed && A == nullptr) return -5;
+  if (lda < std::max(1, m)) return -6;
+  if (work_needed && tau == nullptr) return -7;
+  if (!work_needed) return BQR_SUCCESS;
+  if (!wy_supported(dtype, m, n, lda) || (reinterpret_cast<uintptr_t>(A) & 15))
+    return bqr_geqrf_batched(dtype, m, n, batch, A, lda, tau, stream);  // no blocked variant for this shape
+  if (work == nullptr) return -8;
+  if (work_bytes < wy_workspace_bytes(m, n, 1, kWyPanel)) return -9;
+  return geqrf_wy(m, n, batch, A, lda, tau, work, work_bytes, kWyPanel, stream, &pick_c64_panel);
 }
 
 int bqr_class_count(void) {
@@ -310,10 +398,18 @@ int bqr_geqrf_launches(bqr_dtype_t dtype, int m, int n, int batch) {
   if (geqrf_plan(dtype, m, n, &p)) return 1;
   int nb;
   if (!tiled_panel_width(dtype, m, n, &nb)) return 0;
-  int launches = 0;
+  const bool wy = wy_supported(dtype, m, n, m) && !forced_variant();
   const int kmax = std::min(m, n);
-  for (int k0 = 0; k0 < kmax; k0 += nb) launches += (n - k0 - std::min(nb, kmax - k0) > 0) ? 2 : 1;
-  return launches;
+  // per panel: tiled = panel + apply; WY = panel + V extraction + 4 GEMMs + xLARFT
+  // (one chunk when the batch fits the default path's workspace)
+  const long long chunks =
+      wy ? (batch + std::max<long long>(1, (long long)(kWyMaxWorkspace / wy_workspace_bytes(m, n, 1, kWyPanel))) - 1) /
+               std::max<long long>(1, (long long)(kWyMaxWorkspace / wy_workspace_bytes(m, n, 1, kWyPanel)))
+         : 1;
+  int launches = 0;
+  for (int k0 = 0; k0 < kmax; k0 += nb)
+    launches += (n - k0 - std::min(nb, kmax - k0) > 0) ? (wy ? 7 : 2) : 1;
+  return (int)(launches * chunks);
 }
 
 int bqr_geqrf_batched(bqr_dtype_t dtype, int m, int n, int batch, void *A, int lda, void *tau,
@@ -333,8 +429,12 @@ int bqr_geqrf_batched(bqr_dtype_t dtype, int m, int n, int batch, void *A, int l
   Plan p;
   if (!geqrf_plan(dtype, m, n, &p)) {
     int nb;
-    if (tiled_panel_width(dtype, m, n, &nb)) return geqrf_tiled(dtype, m, n, batch, A, lda, tau, nb, stream);
-    return BQR_ERR_NOT_SUPPORTED;
+    if (!tiled_panel_width(dtype, m, n, &nb)) return BQR_ERR_NOT_SUPPORTED;
+    if (wy_default(dtype, m, n, lda, A) && !forced_variant()) {
+      const int st = geqrf_wy_default(m, n, batch, A, lda, tau, stream);
+      if (st != BQR_ERR_NOT_SUPPORTED) return st;
+    }
+    return geqrf_tiled(dtype, m, n, batch, A, lda, tau, nb, stream);
   }
   Call c{A, tau, batch, m, n, std::min(m, n), lda, stream};
   return p.geqrf(c);

@@ -526,9 +526,13 @@ struct RfKernel {
 #ifndef BQR_FFMA2
 #define BQR_FFMA2 1
 #endif
-  // real classes with the largest register tiles (C3's 14x14 per lane) lose
-  // more to register-pair moves and spills than they gain (measured)
-  static constexpr bool kPacked = BQR_FFMA2 != 0 && (X::kComplex || MR * NC <= 128);
+  // real tiles: packed across column pairs (BQR_FFMA2_COLS; C3 92.0 -> 90.2 us,
+  // f32 128 131.9 -> 127.3 us, profiles/r02/experiments/ab_cols.jsonl)
+#ifndef BQR_FFMA2_COLS
+#define BQR_FFMA2_COLS 1
+#endif
+  static constexpr bool kColPairs = BQR_FFMA2_COLS != 0 && !X::kComplex;
+  static constexpr bool kPacked = BQR_FFMA2 != 0 && (X::kComplex || MR * NC <= 128 || kColPairs);
 
   static __device__ __forceinline__ float2 pk(float x, float y) { return make_float2(x, y); }
 
@@ -609,6 +613,77 @@ struct RfKernel {
     }
   }
 
+  // Real, packed across COLUMN pairs (a[i][2q], a[i][2q+1]) at even absolute
+  // slot indices (the same pairing in every panel, so the register allocator
+  // can keep each pair in an aligned register pair): w_{2q,2q+1} += v_i (a,a'),
+  // (a, a') -= v_i (t_{2q}, t_{2q+1}) with v_i as the FFMA2 scalar operand.
+  // An odd leading / trailing slot of [J0, J1) runs scalar.
+  template <int P, int I0, int J0, int J1>
+  static __device__ __forceinline__ void apply_pk_real_cols(Ctx &c, float (&a)[MR][NC], const float *vb, float ct,
+                                                            int kk, bool skip0 = false) {
+    constexpr int NS = J1 - J0;
+    constexpr bool HEADJ = (J0 & 1) != 0;            // slot J0 unpaired
+    constexpr int JP = HEADJ ? J0 + 1 : J0;          // first paired slot
+    constexpr int NP = (J1 - JP) / 2;                // pairs (JP + 2q, JP + 2q + 1)
+    constexpr bool TAILJ = ((J1 - JP) & 1) != 0;     // slot J1 - 1 unpaired
+    float2 w2[NP > 0 ? NP : 1];
+    float wh = 0.f, wt = 0.f;
+#pragma unroll
+    for (int q = 0; q < (NP > 0 ? NP : 1); ++q) w2[q] = pk(0.f, 0.f);
+    {
+      float v[MR];
+      load_v<I0>(vb, v);
+#pragma unroll
+      for (int i = I0; i < MR; ++i) {
+#pragma unroll
+        for (int q = 0; q < NP; ++q)
+          w2[q] = __ffma2_rn(pk(v[i], v[i]), pk(a[i][JP + 2 * q], a[i][JP + 2 * q + 1]), w2[q]);
+        if constexpr (HEADJ) wh = fmaf(v[i], a[i][J0], wh);
+        if constexpr (TAILJ) wt = fmaf(v[i], a[i][J1 - 1], wt);
+      }
+    }
+    float sum[NS];
+    if constexpr (HEADJ) sum[0] = wh;
+#pragma unroll
+    for (int q = 0; q < NP; ++q) {
+      sum[JP - J0 + 2 * q] = w2[q].x;
+      sum[JP - J0 + 2 * q + 1] = w2[q].y;
+    }
+    if constexpr (TAILJ) sum[NS - 1] = wt;
+    if constexpr (R >= 8 && NS >= 2) {
+      row_allreduce_multi<R, NS>(sum, c.lane);
+    } else {
+#pragma unroll
+      for (int j = 0; j < NS; ++j) sum[j] = row_allreduce<R>(sum[j]);
+    }
+    float tw[NS];
+#pragma unroll
+    for (int j = 0; j < NS; ++j) {
+      tw[j] = ct * sum[j];
+      if (J0 + j == P) tw[j] = c.cg > kk ? tw[j] : 0.f;
+      if (j == 0) tw[j] = skip0 ? 0.f : tw[j];
+    }
+    {
+      float v[MR];
+      load_v<I0>(vb, v);
+#pragma unroll
+      for (int q = 0; q < NP; ++q) {
+        const float2 nt = pk(-tw[JP - J0 + 2 * q], -tw[JP - J0 + 2 * q + 1]);
+#pragma unroll
+        for (int i = I0; i < MR; ++i) {
+          const float2 r = __ffma2_rn(pk(v[i], v[i]), nt, pk(a[i][JP + 2 * q], a[i][JP + 2 * q + 1]));
+          a[i][JP + 2 * q] = r.x;
+          a[i][JP + 2 * q + 1] = r.y;
+        }
+      }
+#pragma unroll
+      for (int i = I0; i < MR; ++i) {
+        if constexpr (HEADJ) a[i][J0] = fmaf(-v[i], tw[0], a[i][J0]);
+        if constexpr (TAILJ) a[i][J1 - 1] = fmaf(-v[i], tw[NS - 1], a[i][J1 - 1]);
+      }
+    }
+  }
+
   // Complex: conj(v) a = (vr, vr) * (ar, ai) + (vi, vi) * (ar, ai) recombined
   // as (A.x + B.y, A.y - B.x); the update a -= v t is
   // a = fma2((vr, vr), (-tr, -ti), a); a = fma2((vi, vi), (ti, -tr), a).
@@ -672,6 +747,8 @@ struct RfKernel {
   static __device__ __forceinline__ void apply_pk(Ctx &c, T (&a)[MR][NC], const T *vb, T ct, int kk, bool skip0) {
     if constexpr (X::kComplex)
       apply_pk_cplx<P, I0, J0, J1>(c, a, vb, ct, kk, skip0);
+    else if constexpr (kColPairs)
+      apply_pk_real_cols<P, I0, J0, J1>(c, a, vb, ct, kk, skip0);
     else
       apply_pk_real<P, I0, J0, J1>(c, a, vb, ct, kk, skip0);
   }

@@ -114,10 +114,20 @@ def test_dispatch(lib, dt, m, n, expect):
     assert bqr.geqrf_launches(dt, m, n, 10) == 1
 
 
-@pytest.mark.parametrize("dt,n,launches", [(1, 256, 5), (1, 192, 3), (1, 176, 3)])
-def test_tiled_dispatch(lib, dt, n, launches):
+@pytest.mark.parametrize("dt,n,launches", [(1, 256, 15), (1, 192, 8), (1, 176, 8)])
+def test_blocked_dispatch(lib, dt, n, launches):
     """Complex shapes above every single-SM class (c64 > 160: more words than
-    one SM's register file) run as tiled panels."""
+    one SM's register file) run the compact-WY blocked variant:
+    per 96-column panel the register-file panel kernel, V extraction, four
+    tensor-core GEMMs and xLARFT (7 launches) when trailing columns remain."""
+    assert bqr.kernel_name(dt, n, n).startswith("wy_c64_panel96")
+    assert bqr.geqrf_launches(dt, n, n, 10) == launches
+
+
+@pytest.mark.parametrize("dt,n,launches", [(1, 255, 5), (1, 177, 3)])
+def test_tiled_dispatch(lib, dt, n, launches):
+    """Odd row counts (16-byte TMA rows impossible) keep the tiled panels:
+    the register-file panel kernel + the Q^H B apply kernel per panel."""
     assert bqr.kernel_name(dt, n, n).startswith("tiled")
     assert bqr.geqrf_launches(dt, n, n, 10) == launches
 
