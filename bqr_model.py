@@ -171,9 +171,10 @@ C4_LAYOUT = Layout(m=240, n=66, R=32, G=11, MR=8, NC=6, cplx=True, resident=1, w
 # 98, named barrier (64 threads) 29, __syncthreads 16 (32 thr) .. 77 (1024),
 # cluster barrier 355-379, DSMEM remote load 202-226; FP32 pipe at 8-16
 # resident warps: FFMA 92, FFMA2 83-88 FMA / clk / SM (of 128); shared
-# memory 127.5 B / clk / SM (Table II analogue).
+# memory 127.5 B / clk / SM (Table II analogue); an empty kernel between two
+# CUDA events 4.96 us (min), 6.9 us (mean).
 B200_R2 = dict(l_fma=4.43, l_shfl_add=30.33, l_lds=29.02, l_sqrtdiv=122.0, l_mbar=98.0, f_ghz=1.965,
-               schedulers=4, fma_per_clk_sm=92.0)
+               schedulers=4, fma_per_clk_sm=92.0, launch_event_us=4.96)
 
 
 def bounds_us(L: Layout, batch: int, instr_total: float, cpi_warp: float, useful_fmas: float,
@@ -192,7 +193,8 @@ def bounds_us(L: Layout, batch: int, instr_total: float, cpi_warp: float, useful
          one included, nothing of the chain hidden.
     The per-matrix latency floor (batch 1, the strong-scaling limit) is the
     chain plus one warp's instructions at CPI 1 (lo1) ... at the measured
-    CPI (hi1)."""
+    CPI (hi1).  The hi bounds add the measured launch / event overhead of an
+    event-timed kernel (B200_R2["launch_event_us"])."""
     f = lat["f_ghz"] * 1e3
     slots = L.resident * n_sm
     rounds = batch / slots
@@ -204,10 +206,13 @@ def bounds_us(L: Layout, batch: int, instr_total: float, cpi_warp: float, useful
     fma = useful_fmas / (lat["fma_per_clk_sm"] * n_sm)
     lo = max(issue, fma, math.ceil(rounds - 1e-9) * chain)
     hi = math.ceil(rounds - 1e-9) * (chain + per_warp_round * cpi_warp)
-    return {"rounds": rounds, "lo_us": lo / f, "hi_us": hi / f,
+    # an event-timed launch also carries the launch / event overhead (an
+    # empty kernel measures 4.96 us min between two CUDA events on B200)
+    return {"rounds": rounds, "lo_us": lo / f, "hi_us": hi / f + lat["launch_event_us"],
             "lo_terms_us": {"issue": issue / f, "fp32_pipe": fma / f, "chain": math.ceil(rounds - 1e-9) * chain / f},
             "chain_cycles_per_matrix": chain, "instr_per_warp_round": per_warp_round, "cpi_warp": cpi_warp,
-            "latency_floor_us": {"lo": (chain + per_warp_round) / f, "hi": (chain + per_warp_round * cpi_warp) / f}}
+            "latency_floor_us": {"lo": (chain + per_warp_round) / f,
+                                 "hi": (chain + per_warp_round * cpi_warp) / f + lat["launch_event_us"]}}
 
 
 S80_LAYOUT = Layout(m=80, n=16, R=16, G=4, MR=5, NC=4, cplx=True, resident=8, warps_per_matrix=2,

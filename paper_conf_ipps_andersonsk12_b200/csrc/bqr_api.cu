@@ -155,14 +155,25 @@ bool tiled_panel_width(bqr_dtype_t dt, int m, int n, int *nb) {
   return n > *nb;
 }
 
-// compact-WY blocked variant (bqr_wy.cu) for the complex shapes beyond one
-// SM: 96-column register panels + tensor-core trailing updates
+// compact-WY blocked variant (bqr_wy.cu): register-file panels (64 fp32 /
+// 96 complex columns) + tensor-core trailing updates
 const Plan *pick_c64_panel(int m, int n) { return pick(BQR_C64, m, n); }
-constexpr int kWyPanel = 96;
+const Plan *pick_f32_panel(int m, int n) { return pick(BQR_R32, m, n); }
 constexpr size_t kWyMaxWorkspace = size_t(2) << 30;  // stream-ordered workspace cap of the default path
 
+const char *wy_name(bqr_dtype_t dt) {
+  return dt == BQR_R32 ? "wy_f32_panel64+tcgen05_fastf32_gemm" : "wy_c64_panel96+tcgen05_fastf32_gemm";
+}
+
+// shapes bqr_geqrf_batched itself factors with the blocked variant: the
+// complex ones beyond every single-SM class (measured 1.4-1.8x faster than
+// the tiled panels, profiles/r02/experiments/wy_vs_tiled.jsonl)
+bool wy_default_shape(bqr_dtype_t dt, int m, int n, int lda) {
+  return dt == BQR_C64 && n > 160 && wy_supported(dt, m, n, lda) && !forced_variant();
+}
+
 bool wy_default(bqr_dtype_t dt, int m, int n, int lda, const void *A) {
-  return wy_supported(dt, m, n, lda) && (reinterpret_cast<uintptr_t>(A) & 15) == 0;
+  return wy_default_shape(dt, m, n, lda) && (reinterpret_cast<uintptr_t>(A) & 15) == 0;
 }
 
 // a library-private stream-ordered memory pool per device that keeps its
@@ -194,17 +205,19 @@ cudaMemPool_t wy_pool() {
 // caller's stream (cudaMallocFromPoolAsync / cudaFreeAsync: no host
 // synchronisation, private to this call); the tiled path if the pool cannot
 // provide it
-int geqrf_wy_default(int m, int n, long long batch, void *A, int lda, void *tau, cudaStream_t stream) {
-  const size_t per = wy_workspace_bytes(m, n, 1, kWyPanel);
+int geqrf_wy_default(bqr_dtype_t dt, int m, int n, long long batch, void *A, int lda, void *tau,
+                     cudaStream_t stream) {
+  const size_t per = wy_workspace_bytes(dt, m, n, 1);
   const long long chunk = std::max<long long>(1, std::min<long long>(batch, (long long)(kWyMaxWorkspace / per)));
-  const size_t bytes = wy_workspace_bytes(m, n, (int)chunk, kWyPanel);
+  const size_t bytes = wy_workspace_bytes(dt, m, n, (int)chunk);
   cudaMemPool_t pool = wy_pool();
   void *ws = nullptr;
   if (!pool || cudaMallocFromPoolAsync(&ws, bytes, pool, stream) != cudaSuccess) {
     cudaGetLastError();
     return BQR_ERR_NOT_SUPPORTED;
   }
-  const int st = geqrf_wy(m, n, batch, A, lda, tau, ws, bytes, kWyPanel, stream, &pick_c64_panel);
+  const int st = geqrf_wy(dt, m, n, batch, A, lda, tau, ws, bytes, stream,
+                          dt == BQR_R32 ? &pick_f32_panel : &pick_c64_panel);
   cudaFreeAsync(ws, stream);
   return st;
 }
@@ -319,8 +332,7 @@ const char *bqr_kernel_name(bqr_dtype_t dtype, int m, int n) {
   if (!geqrf_plan(dtype, m, n, &p)) {
     int nb;
     if (!tiled_panel_width(dtype, m, n, &nb)) return "";
-    return (wy_supported(dtype, m, n, m) && !forced_variant()) ? "wy_c64_panel96+tcgen05_fastf32_gemm"
-                                                              : "tiled_c64_panel96+apply";
+    return wy_default_shape(dtype, m, n, m) ? wy_name(dtype) : "tiled_c64_panel96+apply";
   }
   return p.name ? p.name : "";
 }
@@ -340,13 +352,13 @@ long long bqr_resident_matrices(bqr_dtype_t dtype, int m, int n) {
 size_t bqr_geqrf_wy_workspace_bytes(bqr_dtype_t dtype, int m, int n, int lda, int chunk) {
   if (!valid_dtype(dtype) || m <= 0 || n <= 0 || chunk <= 0) return 0;
   if (!wy_supported(dtype, m, n, lda)) return 0;
-  return wy_workspace_bytes(m, n, chunk, kWyPanel);
+  return wy_workspace_bytes(dtype, m, n, chunk);
 }
 
 const char *bqr_geqrf_wy_kernel_name(bqr_dtype_t dtype, int m, int n, int lda) {
   if (!valid_dtype(dtype) || m <= 0 || n <= 0 || m < n) return "";
   if (!wy_supported(dtype, m, n, lda)) return bqr_kernel_name(dtype, m, n);
-  return "wy_c64_panel96+tcgen05_fastf32_gemm";
+  return wy_name(dtype);
 }
 
 int bqr_geqrf_wy_batched(bqr_dtype_t dtype, int m, int n, int batch, void *A, int lda, void *tau, void *work,
@@ -363,8 +375,9 @@ int bqr_geqrf_wy_batched(bqr_dtype_t dtype, int m, int n, int batch, void *A, in
   if (!wy_supported(dtype, m, n, lda) || (reinterpret_cast<uintptr_t>(A) & 15))
     return bqr_geqrf_batched(dtype, m, n, batch, A, lda, tau, stream);  // no blocked variant for this shape
   if (work == nullptr) return -8;
-  if (work_bytes < wy_workspace_bytes(m, n, 1, kWyPanel)) return -9;
-  return geqrf_wy(m, n, batch, A, lda, tau, work, work_bytes, kWyPanel, stream, &pick_c64_panel);
+  if (work_bytes < wy_workspace_bytes(dtype, m, n, 1)) return -9;
+  return geqrf_wy(dtype, m, n, batch, A, lda, tau, work, work_bytes, stream,
+                  dtype == BQR_R32 ? &pick_f32_panel : &pick_c64_panel);
 }
 
 int bqr_class_count(void) {
@@ -398,14 +411,13 @@ int bqr_geqrf_launches(bqr_dtype_t dtype, int m, int n, int batch) {
   if (geqrf_plan(dtype, m, n, &p)) return 1;
   int nb;
   if (!tiled_panel_width(dtype, m, n, &nb)) return 0;
-  const bool wy = wy_supported(dtype, m, n, m) && !forced_variant();
+  const bool wy = wy_default_shape(dtype, m, n, m);
   const int kmax = std::min(m, n);
   // per panel: tiled = panel + apply; WY = panel + V extraction + 4 GEMMs + xLARFT
   // (one chunk when the batch fits the default path's workspace)
-  const long long chunks =
-      wy ? (batch + std::max<long long>(1, (long long)(kWyMaxWorkspace / wy_workspace_bytes(m, n, 1, kWyPanel))) - 1) /
-               std::max<long long>(1, (long long)(kWyMaxWorkspace / wy_workspace_bytes(m, n, 1, kWyPanel)))
-         : 1;
+  const long long per_chunk =
+      wy ? std::max<long long>(1, (long long)(kWyMaxWorkspace / wy_workspace_bytes(dtype, m, n, 1))) : batch;
+  const long long chunks = (batch + per_chunk - 1) / per_chunk;
   int launches = 0;
   for (int k0 = 0; k0 < kmax; k0 += nb)
     launches += (n - k0 - std::min(nb, kmax - k0) > 0) ? (wy ? 7 : 2) : 1;
@@ -431,7 +443,7 @@ int bqr_geqrf_batched(bqr_dtype_t dtype, int m, int n, int batch, void *A, int l
     int nb;
     if (!tiled_panel_width(dtype, m, n, &nb)) return BQR_ERR_NOT_SUPPORTED;
     if (wy_default(dtype, m, n, lda, A) && !forced_variant()) {
-      const int st = geqrf_wy_default(m, n, batch, A, lda, tau, stream);
+      const int st = geqrf_wy_default(dtype, m, n, batch, A, lda, tau, stream);
       if (st != BQR_ERR_NOT_SUPPORTED) return st;
     }
     return geqrf_tiled(dtype, m, n, batch, A, lda, tau, nb, stream);

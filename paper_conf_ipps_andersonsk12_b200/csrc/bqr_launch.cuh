@@ -205,9 +205,10 @@ int apply_dispatch_f32(const ApplyArgs &a, cudaStream_t s);
 int apply_dispatch_c64(const ApplyArgs &a, cudaStream_t s);
 int launch_selftest_math(long long n, unsigned seed, unsigned long long *counts, cudaStream_t s);
 // compact-WY blocked QR with tensor-core trailing updates (bqr_wy.cu)
+int wy_panel_width(bqr_dtype_t dt);
 bool wy_supported(bqr_dtype_t dt, int m, int n, int lda);
-size_t wy_workspace_bytes(int m, int n, int chunk, int nb);
-int geqrf_wy(int m, int n, long long batch, void *A, int lda, void *tau, void *work, size_t work_bytes, int nb,
+size_t wy_workspace_bytes(bqr_dtype_t dt, int m, int n, int chunk);
+int geqrf_wy(bqr_dtype_t dt, int m, int n, long long batch, void *A, int lda, void *tau, void *work, size_t work_bytes,
              cudaStream_t stream, const Plan *(*pick_panel)(int, int));
 // back substitution X = R^{-1} C of the least-squares path (bqr_solve.cu)
 int solve_upper_dispatch(bqr_dtype_t dt, const void *A, int lda, long long strideA, void *B, int ldb,

@@ -24,16 +24,17 @@ def wy_gpu(A_cm, m, chunk=None):
     buf = torch.from_numpy(np.ascontiguousarray(A_cm)).cuda()
     tau = torch.full((batch, min(m, n)), float("nan"), dtype=buf.dtype, device="cuda")
     chunk = batch if chunk is None else chunk
-    wsb = max(1, bqr.geqrf_wy_workspace_bytes(bqr.C64, m, n, lda, chunk))
+    code = bqr.C64 if np.iscomplexobj(A_cm) else bqr.R32
+    wsb = max(1, bqr.geqrf_wy_workspace_bytes(code, m, n, lda, chunk))
     ws = torch.empty(wsb, dtype=torch.uint8, device="cuda")
-    st = bqr.geqrf_wy_batched_ptr(bqr.C64, m, n, batch, buf.data_ptr(), lda, tau.data_ptr(), ws.data_ptr(), wsb)
+    st = bqr.geqrf_wy_batched_ptr(code, m, n, batch, buf.data_ptr(), lda, tau.data_ptr(), ws.data_ptr(), wsb)
     assert st == 0, bqr.load().bqr_status_string(st)
     torch.cuda.synchronize()
     return buf.cpu().numpy(), tau.cpu().numpy()
 
 
 @pytest.mark.parametrize("m,n", [(192, 192), (224, 224), (256, 256), (256, 200), (176, 176), (256, 161),
-                                 (240, 180)])
+                                 (240, 180), (128, 128), (160, 160), (98, 97)])
 def test_wy_parity(m, n):
     assert "tcgen05" in bqr.load().bqr_geqrf_wy_kernel_name(bqr.C64, m, n, m).decode()
     A = bqr_inputs.random_batch(m, n, 24, "c64", seed=5000 + m + n)
@@ -41,6 +42,16 @@ def test_wy_parity(m, n):
     rep = compare_geqrf(A, m, out, tau, full_q=False)
     assert rep["ok"], rep
     assert rep["residual_max"] < 3e-6 and rep["orth_max"] < 5e-6, rep
+
+
+@pytest.mark.parametrize("m,n", [(256, 256), (192, 192), (224, 224), (128, 128), (96, 96), (256, 100), (200, 65)])
+def test_wy_parity_f32(m, n):
+    """fp32: 64-column register panels + real FastF32 tensor-core GEMMs."""
+    assert "wy_f32_panel64" in bqr.load().bqr_geqrf_wy_kernel_name(bqr.R32, m, n, m).decode()
+    A = bqr_inputs.random_batch(m, n, 24, "f32", seed=6000 + m + n)
+    out, tau = wy_gpu(A, m)
+    rep = compare_geqrf(A, m, out, tau, full_q=m <= 128)
+    assert rep["ok"], rep
 
 
 def test_wy_chunked_and_deterministic():
@@ -56,16 +67,20 @@ def test_wy_chunked_and_deterministic():
 
 
 def test_wy_forwards_unsupported_shapes():
-    """Shapes without a blocked variant (real, n <= 160) take bqr_geqrf_batched."""
-    A = bqr_inputs.random_batch(128, 128, 8, "c64", seed=72)
-    out, tau = wy_gpu(A, 128)
-    assert compare_geqrf(A, 128, out, tau, full_q=False)["ok"]
-    assert bqr.load().bqr_geqrf_wy_kernel_name(bqr.C64, 128, 128, 128).decode() == bqr.kernel_name(bqr.C64, 128, 128)
+    """Shapes without a blocked variant (one panel wide, or rows that are not
+    a 16-byte multiple) take bqr_geqrf_batched."""
+    for m, n, dt in ((64, 64, "c64"), (99, 97, "c64"), (130, 130, "f32")):
+        A = bqr_inputs.random_batch(m, n, 8, dt, seed=72)
+        out, tau = wy_gpu(A, m)
+        assert compare_geqrf(A, m, out, tau, full_q=False)["ok"]
+        code = bqr.C64 if dt == "c64" else bqr.R32
+        assert bqr.load().bqr_geqrf_wy_kernel_name(code, m, n, m).decode() == bqr.kernel_name(code, m, n)
 
 
-@pytest.mark.parametrize("kind", ["graded", "near_rank"])
-def test_wy_contract_edges(kind):
-    A = bqr_inputs.stress_batch(256, 256, 6, "c64", kind, seed=73)
+@pytest.mark.parametrize("dt", ["c64", "f32"])
+@pytest.mark.parametrize("kind", ["graded", "near_rank", "tiny", "huge"])
+def test_wy_contract_edges(kind, dt):
+    A = bqr_inputs.stress_batch(256, 256, 6, dt, kind, seed=73)
     out, tau = wy_gpu(A, 256)
     rep = compare_geqrf(A, 256, out, tau, full_q=False)
     assert rep["ok"], {k: v for k, v in rep.items() if k != "fail_idx"}

@@ -327,6 +327,11 @@ __global__ void k_dsmem_chase(float *out, long long *cyc, int iters) {
   if (threadIdx.x == 0 && cl.block_rank() == 0) cyc[0] = t1 - t0;
 }
 
+// ---------------------------------------------------------------- launch overhead
+__global__ void k_empty(float *out) {
+  if (out && threadIdx.x == 1023) out[0] = 0.f;
+}
+
 // ---------------------------------------------------------------- host
 static unsigned long long max_cyc(int nblk) {
   static unsigned long long h[4096];
@@ -417,6 +422,34 @@ int main() {
     cudaLaunchKernelEx(&cfg, k_dsmem_chase, out, cyc, iters);
     cudaMemcpy(&h, cyc, 8, cudaMemcpyDeviceToHost);
     printf("{\"bench\":\"dsmem_remote_load_latency\",\"cluster\":%d,\"cycles\":%.2f}\n", cs, h / (iters * 16.0));
+  }
+  {  // CUDA-event time of an empty launch (what an event-timed kernel adds)
+    cudaEvent_t a, b2;
+    cudaEventCreate(&a);
+    cudaEventCreate(&b2);
+    float best = 1e9, sum = 0.f;
+    for (int r = 0; r < 200; ++r) {
+      cudaEventRecord(a);
+      k_empty<<<1, 32>>>(nullptr);
+      cudaEventRecord(b2);
+      cudaEventSynchronize(b2);
+      float ms;
+      cudaEventElapsedTime(&ms, a, b2);
+      if (r >= 20) {
+        best = ms < best ? ms : best;
+        sum += ms;
+      }
+    }
+    printf("{\"bench\":\"empty_launch_event_us\",\"min\":%.2f,\"mean\":%.2f}\n", best * 1e3, sum / 180 * 1e3);
+    for (int r = 0; r < 3; ++r) {
+      cudaEventRecord(a);
+      k_empty<<<148 * 8, 64>>>(nullptr);
+      cudaEventRecord(b2);
+      cudaEventSynchronize(b2);
+    }
+    float ms;
+    cudaEventElapsedTime(&ms, a, b2);
+    printf("{\"bench\":\"empty_grid_1184x64_event_us\",\"value\":%.2f}\n", ms * 1e3);
   }
   cudaError_t e = cudaDeviceSynchronize();
   printf("{\"sms\":%d,\"clock_khz\":%d,\"status\":\"%s\"}\n", sms, clk, cudaGetErrorString(e));

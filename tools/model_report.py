@@ -1,40 +1,66 @@
 """NEXT-4 report: the paper's Table VI model (Fermi parameters) against its
-Table V measurements, and the B200 re-parameterisation (bqr_model) against
-this round's measurements (profiles/bench_r01.json, phase timer).  Writes
-profiles/model_r01.json.
+Table V measurements, and the B200 bounds of bqr_model.bounds_us (measured
+microbenchmark latencies + this round's ncu instruction counts and warp CPI)
+against this round's bench times and batch-1 latencies.  Writes
+profiles/model_r02.json.
 
-    python tools/model_report.py
+    python tools/model_report.py [bench.json]
 """
 import json
 import os
+import re
 import sys
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
+import bqr_metrics as bm  # noqa: E402
 import bqr_model as M  # noqa: E402
+
+NCU = os.path.join(ROOT, "profiles", "r02", "ncu")
+
+
+def ncu_metric(cfg: str, name: str) -> float:
+    with open(os.path.join(NCU, f"details_{cfg}.txt")) as f:
+        for line in f:
+            if line.startswith(name):
+                return float(re.findall(r"[-+]?\d[\d.]*", line[len(name):])[0])
+    raise KeyError(name)
 
 
 def main():
-    bench = json.load(open(os.path.join(ROOT, "profiles", "bench_r01.json")))
+    bench_path = sys.argv[1] if len(sys.argv) > 1 else os.path.join(ROOT, "profiles", "r02", "bench_r02b.json")
+    bench = json.load(open(bench_path))
     out = {"paper_fermi": {
         "qr_56": {"model_cycles": M.paper_qr_cycles(56), "paper_measured_cycles": 150203},
         "lu_56": {"model_cycles": M.paper_lu_cycles(56), "paper_measured_cycles": 68250},
-        "readings": "b = shared latency 27, g = 18, a_sync = 46 (Table IV); g_sqrt = g_div = 2 g (not printed)"}}
-    c3 = M.predict_us(M.C3_LAYOUT, 5000)
-    c3["measured_us"] = bench["roofline"]["kernel_us"]
-    c4 = M.predict_us(M.C4_LAYOUT, 256)
-    c4["measured_us_fused_step"] = bench["also"]["C4"]["roofline"]["kernel_us"]
-    one = M.predict_us(M.C4_LAYOUT, 1)
-    ph = os.path.join(ROOT, "profiles", "r01", "experiments", "ph_c4_dec_1.jsonl")
-    if os.path.exists(ph):
-        rows = [json.loads(line) for line in open(ph) if line.startswith("{")]
-        one["measured_step_cycles_phase_timer"] = rows[-1].get("total_cycles")
-    one["model_chain_plus_issue_cycles"] = one["chain_cycles"] + one["issue_cycles"]
-    out["b200"] = {"C3": c3, "C4": c4, "C4_one_matrix": one,
-                   "note": "lo = perfect overlap of the reflector chain with the trailing update at IPC 1 per "
-                           "scheduler, hi = no overlap; measured above hi = issue stalls the model does not "
-                           "price (FMA dependency waits, register-bank dispatch stalls, ncu 'wait'/'dispatch')"}
-    path = os.path.join(ROOT, "profiles", "model_r01.json")
+        "readings": "b = shared latency 27, g = 18, a_sync = 46 (Table IV); g_sqrt = g_div = 2 g (not printed)"},
+        "b200": {}}
+    cases = {
+        "C3": (M.C3_LAYOUT, 5000, bench["roofline"]["kernel_us"], bench["latency"]["batch_1_us"], 56, 56, "f32"),
+        "C4": (M.C4_LAYOUT, 256, bench["also"]["C4"]["roofline"]["kernel_us"],
+               bench["also"]["C4"].get("latency", {}).get("batch_1_us"), 240, 66, "c64"),
+        "S80": (M.S80_LAYOUT, 384, bench["also"]["S80"]["roofline"]["kernel_us"], None, 80, 16, "c64"),
+    }
+    for cfg, (L, batch, measured, lat1, m, n, dt) in cases.items():
+        instr = ncu_metric(cfg, "Executed Instructions")
+        cpi = ncu_metric(cfg, "Warp Cycles Per Issued Instruction")
+        fmas = batch * bm.geqrf_flops(m, n, dt) / 2
+        if cfg == "C4":  # the bench step is the fused [A | b] factorisation
+            fmas += batch * bm.apply_flops(m, n, 1, dt) / 2
+        b = M.bounds_us(L, batch, instr, cpi, fmas)
+        b["measured_us"] = measured
+        b["bracketed"] = bool(b["lo_us"] <= measured <= b["hi_us"])
+        if lat1 is not None:
+            b["latency_floor_us"]["measured_batch_1"] = lat1
+            b["latency_floor_us"]["bracketed"] = bool(b["latency_floor_us"]["lo"] <= lat1 <= b["latency_floor_us"]["hi"])
+        b["ncu"] = {"executed_instructions": instr, "warp_cpi": cpi}
+        out["b200"][cfg] = b
+    out["b200"]["note"] = ("lo = max(issue of every executed warp instruction at 1 / scheduler / cycle, useful FMAs at "
+                           "the measured FFMA rate, rounds x the per-matrix reflector chain); hi = ceil(rounds) x "
+                           "(chain + one warp's instructions per round x the measured warp CPI); latency floor = "
+                           "chain + one warp's instructions at CPI 1 .. at the measured CPI.  Constants: "
+                           "profiles/r02/micro2.jsonl (tools/micro/micro2.cu); counts: profiles/r02/ncu/details_*.txt.")
+    path = os.path.join(ROOT, "profiles", "model_r02.json")
     with open(path, "w") as f:
         json.dump(out, f, indent=1)
     print(json.dumps(out, indent=1))

@@ -19,30 +19,35 @@ import bqr_metrics as bm  # noqa: E402
 import paper_conf_ipps_andersonsk12_b200 as bqr  # noqa: E402
 from oracle.compare import compare_geqrf  # noqa: E402
 
-sizes = [int(x) for x in sys.argv[1:]] or [176, 192, 224, 256]
+args = sys.argv[1:]
+cells = []
+for a in args or ["c64:176", "c64:192", "c64:224", "c64:256"]:
+    dt, n = (a.split(":") if ":" in a else ("c64", a))
+    cells.append((dt, int(n)))
 n_sm = torch.cuda.get_device_properties(0).multi_processor_count
 flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
 peaks = bm.load_peaks()
-for n in sizes:
-    cfg = bqr_inputs.c5_config(n, "c64", n_sm=n_sm)
+for dt, n in cells:
+    code = bqr.C64 if dt == "c64" else bqr.R32
+    cfg = bqr_inputs.c5_config(n, dt, n_sm=n_sm)
     B = cfg["batch"]
-    A = bqr_inputs.random_batch(n, n, B, "c64", cfg["seed"])
+    A = bqr_inputs.random_batch(n, n, B, dt, cfg["seed"])
     pristine = torch.from_numpy(A).cuda()
     buf = torch.empty_like(pristine)
     tau = torch.empty((B, n), dtype=buf.dtype, device="cuda")
-    wsb = bqr.geqrf_wy_workspace_bytes(bqr.C64, n, n, n, B)
+    wsb = bqr.geqrf_wy_workspace_bytes(code, n, n, n, B)
     ws = torch.empty(max(1, wsb), dtype=torch.uint8, device="cuda")
     s = torch.cuda.current_stream()
 
     def run(kind):
         if kind == "wy":
-            st = bqr.geqrf_wy_batched_ptr(bqr.C64, n, n, B, buf.data_ptr(), n, tau.data_ptr(), ws.data_ptr(), wsb)
+            st = bqr.geqrf_wy_batched_ptr(code, n, n, B, buf.data_ptr(), n, tau.data_ptr(), ws.data_ptr(), wsb)
         else:
-            st = bqr.geqrf_batched_ptr(bqr.C64, n, n, B, buf.data_ptr(), n, tau.data_ptr(), s.cuda_stream)
+            st = bqr.geqrf_batched_ptr(code, n, n, B, buf.data_ptr(), n, tau.data_ptr(), s.cuda_stream)
         assert st == 0, st
 
-    flops = B * bm.geqrf_flops(n, n, "c64")
-    nbytes = B * bm.geqrf_bytes(n, n, "c64")
+    flops = B * bm.geqrf_flops(n, n, dt)
+    nbytes = B * bm.geqrf_bytes(n, n, dt)
     fp32 = bm.fp32_peak_tflops(n_sm, float(peaks.get("sm_max_mhz", 1965.0)))
     t_roof, bound = bm.roofline_time_s(flops, nbytes, float(peaks["hbm_gbs"]), fp32)
     for kind in ("default", "wy"):
@@ -64,8 +69,8 @@ for n in sizes:
         out = buf[torch.from_numpy(idx).cuda()].cpu().numpy()
         tu = tau[torch.from_numpy(idx).cuda()].cpu().numpy()
         rep = compare_geqrf(A[idx], n, out, tu, full_q=False)
-        name = bqr.load().bqr_geqrf_wy_kernel_name(bqr.C64, n, n, n).decode() if kind == "wy" else bqr.kernel_name(bqr.C64, n, n)
-        print(json.dumps({"n": n, "dtype": "c64", "batch": B, "path": kind, "kernel": name, "ms": round(ms, 4),
+        name = bqr.load().bqr_geqrf_wy_kernel_name(code, n, n, n).decode() if kind == "wy" else bqr.kernel_name(code, n, n)
+        print(json.dumps({"n": n, "dtype": dt, "batch": B, "path": kind, "kernel": name, "ms": round(ms, 4),
                           "tflops": round(flops / ms / 1e9, 3), "roofline_frac": round(t_roof / (ms / 1e3), 4),
                           "bound": bound, "parity_ok": rep["ok"], "residual": rep["residual_max"],
                           "orth": rep["orth_max"], "sampled": len(idx)}), flush=True)
