@@ -343,26 +343,38 @@ def e2e_host(w: Workload, steps: int, warmup: int, torch, dist, world):
     return ms, h2d, d2h
 
 
-def cpu_baseline(name: str, min_seconds: float = 3.0, max_matrices: int | None = None):
-    """The fp64 oracle, as it stands, on all host cores, on a bounded sample."""
+def cpu_baseline(name: str, min_seconds: float = 2.0, max_matrices: int | None = None):
+    """The fp64 oracle, as it stands, on a bounded sample: the median of 3
+    timed trials on all host cores, plus one trial on 1 core."""
     import oracle
     cfg = bqr_inputs.CONFIGS[name]
     b = cfg["batch"] if max_matrices is None else min(cfg["batch"], max_matrices)
     A = bqr_inputs.random_batch(cfg["m"], cfg["n"], cfg["batch"], cfg["dtype"], cfg["seed"], cfg["dist"], stop=b)
+    per = bm.geqrf_flops(cfg["m"], cfg["n"], cfg["dtype"])
+
+    def trial(Ab, secs):
+        reps, t0 = 0, time.perf_counter()
+        while True:
+            oracle.geqrf_cm(Ab, cfg["m"], with_margin=False)
+            reps += 1
+            el = time.perf_counter() - t0
+            if el >= secs:
+                return reps * Ab.shape[0] / el  # matrices / s
+
     oracle.set_threads(0)
     oracle.geqrf_cm(A, cfg["m"], with_margin=False)  # warm (page-in, threads)
-    reps, t0 = 0, time.perf_counter()
-    while True:
-        oracle.geqrf_cm(A, cfg["m"], with_margin=False)
-        reps += 1
-        el = time.perf_counter() - t0
-        if el >= min_seconds:
-            break
-    flops = reps * b * bm.geqrf_flops(cfg["m"], cfg["n"], cfg["dtype"])
-    return {"value": round(flops / el / 1e9, 4), "unit": UNIT, "cores": oracle.max_threads(), "kind": "oracle",
-            "sample": f"{b} of the {name} matrices ({cfg['m']}x{cfg['n']} {cfg['dtype']}) x {reps} passes, "
-                      f"{el:.1f} s wall, fp64 C oracle (OpenMP)",
-            "matrices_per_s": round(reps * b / el, 1)}
+    rates = sorted(trial(A, min_seconds / 2) for _ in range(3))
+    cores = oracle.max_threads()
+    oracle.set_threads(1)
+    one = trial(A[: max(1, b // 16)], min_seconds / 4)
+    oracle.set_threads(0)
+    med = rates[1]
+    return {"value": round(med * per / 1e9, 4), "unit": UNIT, "cores": cores, "kind": "oracle",
+            "sample": f"{b} of the {name} matrices ({cfg['m']}x{cfg['n']} {cfg['dtype']}), median of 3 trials of "
+                      f"~{min_seconds / 2:.1f} s on {cores} threads; 1-core trial on {max(1, b // 16)} matrices; "
+                      f"fp64 C oracle (OpenMP)",
+            "matrices_per_s": round(med, 1), "trials_gflops": [round(r * per / 1e9, 4) for r in rates],
+            "value_1core": round(one * per / 1e9, 4)}
 
 
 def config_block(w: Workload, world, l2_note):
@@ -484,7 +496,7 @@ def run_ours(args):
     peaks = bm.load_peaks()
 
     main = Workload(args.config, rank, world, torch, bqr, scaling=args.scaling)
-    sampler = ClockSampler(local)
+    sampler = ClockSampler(local, 0.002)
     step_ms, qr_ms = time_workload(main, args.steps, args.warmup, torch, dist, world, flush, sampler)
     value = main.step_flops_total() / (step_ms / 1e3) / 1e9
     out = {
