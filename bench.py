@@ -384,7 +384,8 @@ def config_block(w: Workload, world, l2_note):
     return {"workload": f"{w.name}: {w.batch} x {w.m}x{w.n} {w.dt} {op} per GPU", "m": w.m, "n": w.n,
             "batch_per_gpu": w.batch, "global_batch": w.global_batch,
             "dtype": w.dt, "l2": l2_note, "parallelism": f"dp{world} (independent matrices per rank)",
-            "kernel": w.bqr.kernel_name(w.code, w.m, w.n) if w.kind == "qr" else "lu_rf_kernel"}
+            "kernel": (w.bqr.load().bqr_qhb_kernel_name(w.code, w.m, w.n, w.nrhs).decode() if w.nrhs and w.kind == "qr"
+                       else w.bqr.kernel_name(w.code, w.m, w.n) if w.kind == "qr" else "lu_rf_kernel")}
 
 
 def latency_scan(w: Workload, torch, dist, world, flush, n_sm: int) -> dict:

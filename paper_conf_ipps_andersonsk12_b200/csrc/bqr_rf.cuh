@@ -272,7 +272,11 @@ struct RfKernel {
   static __device__ __forceinline__ void sig_arrive(Ctx &c, int k) {
     if constexpr (Cfg::LAZY) {
       // every lane of the publishing warp arrives (count 32): each lane's
-      // vector stores are released by its own arrive
+      // vector stores are released by its own arrive; the warp barrier first
+      // orders lane 0's tau store before every lane's arrive (so the release
+      // covers it too -- racecheck cannot otherwise prove the tau read of
+      // the consumers ordered)
+      warp_sync();
       asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(c.full + (c.gbase + k) % NBUF))
                    : "memory");
     } else {

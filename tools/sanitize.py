@@ -102,6 +102,17 @@ def case_host(dt, m, n, batch):
     return f"geqrf_batched_host {dt} {m}x{n} x{batch}"
 
 
+def case_wy(dt, m, n, batch):
+    A = dev(bqr_inputs.random_batch(m, n, batch, dt, seed=11))
+    tau = torch.empty((batch, min(m, n)), dtype=A.dtype, device="cuda")
+    wsb = bqr.geqrf_wy_workspace_bytes(code(dt), m, n, m, batch)
+    ws = torch.empty(wsb, dtype=torch.uint8, device="cuda")
+    st = bqr.geqrf_wy_batched_ptr(code(dt), m, n, batch, A.data_ptr(), m, tau.data_ptr(), ws.data_ptr(), wsb)
+    assert st == 0, ("wy", dt, m, n, st)
+    torch.cuda.synchronize()
+    return f"geqrf_wy {dt} {m}x{n} x{batch}"
+
+
 CASES = [
     (case_geqrf, ("f32", 4, 4, 300)),          # tiny, thread per matrix
     (case_geqrf, ("c64", 8, 8, 100)),
@@ -115,7 +126,10 @@ CASES = [
     (case_geqrf, ("c64", 80, 16, 40)),         # STAP 80x16 warp class
     (case_geqrf, ("c64", 192, 96, 150)),       # STAP 192x96 (R = 32)
     (case_geqrf, ("f32", 256, 256, 4)),        # single-SM 256 class
-    (case_geqrf, ("c64", 224, 224, 3)),        # tiled panels (a9)
+    (case_geqrf, ("c64", 224, 224, 3)),        # compact WY (a6/a9): panels + tcgen05 GEMMs + xLARFT
+    (case_geqrf, ("c64", 225, 225, 3)),        # odd rows: tiled panels (a9)
+    (case_geqrf, ("c64", 112, 112, 20)),       # R16G16 7x7 CTA class (97..112)
+    (case_wy, ("f32", 256, 256, 3)),           # compact WY, fp32, caller workspace
     (case_orgqr_apply, ("f32", 56, 56, 30)),
     (case_orgqr_apply, ("c64", 240, 66, 10)),
     (case_qhb_gels, ("c64", 240, 66, 150)),    # fused augmented class (persistent loop)
@@ -126,7 +140,7 @@ CASES = [
     (case_host, ("f32", 56, 56, 300)),
 ]
 if QUICK:
-    CASES = [c for i, c in enumerate(CASES) if i in (0, 3, 6, 8, 12, 15, 17, 20)]
+    CASES = [c for i, c in enumerate(CASES) if i in (0, 3, 6, 8, 12, 13, 14, 18, 20, 23)]
 
 for fn, args in CASES:
     print("ok", fn(*args), flush=True)
