@@ -22,21 +22,25 @@
 using namespace cute;
 using Cf = cutlass::complex<float>;
 
-template <class LayoutA, class LayoutB>
+template <class LayoutA, class LayoutB, bool TWO_SM = false>
 struct FastGemm {
   using LayoutC = cutlass::layout::ColumnMajor;
-  using MmaTileShape = Shape<_128, _64, _16>;
-  using ClusterShape = Shape<_1, _1, _1>;
+  using MmaTileShape = cute::conditional_t<TWO_SM, Shape<_256, _64, _16>, Shape<_128, _64, _16>>;
+  using ClusterShape = cute::conditional_t<TWO_SM, Shape<_2, _1, _1>, Shape<_1, _1, _1>>;
+  using EpiSched = cute::conditional_t<TWO_SM, cutlass::epilogue::FastF32NoSmemWarpSpecialized2Sm,
+                                       cutlass::epilogue::FastF32NoSmemWarpSpecialized1Sm>;
+  using MainSched = cute::conditional_t<TWO_SM, cutlass::gemm::KernelTmaWarpSpecialized2SmFastFP32Sm100,
+                                        cutlass::gemm::KernelTmaWarpSpecialized1SmFastFP32Sm100>;
   using CollectiveEpilogue = typename cutlass::epilogue::collective::CollectiveBuilder<
       cutlass::arch::Sm100, cutlass::arch::OpClassTensorOp, MmaTileShape, ClusterShape,
       cutlass::epilogue::collective::EpilogueTileAuto, Cf, Cf, Cf, LayoutC, 2, Cf, LayoutC, 2,
-      cutlass::epilogue::FastF32NoSmemWarpSpecialized1Sm>::CollectiveOp;
+      EpiSched>::CollectiveOp;
   using CollectiveMainloop = typename cutlass::gemm::collective::CollectiveBuilder<
       cutlass::arch::Sm100, cutlass::arch::OpClassTensorOp, Cf, LayoutA, 2, Cf, LayoutB, 2, Cf, MmaTileShape,
       ClusterShape,
       cutlass::gemm::collective::StageCountAutoCarveout<static_cast<int>(
           sizeof(typename CollectiveEpilogue::SharedStorage))>,
-      cutlass::gemm::KernelTmaWarpSpecialized1SmFastFP32Sm100>::CollectiveOp;
+      MainSched>::CollectiveOp;
   using Kernel = cutlass::gemm::kernel::GemmUniversal<Shape<int, int, int, int>, CollectiveMainloop,
                                                       CollectiveEpilogue>;
   using Gemm = cutlass::gemm::device::GemmUniversalAdapter<Kernel>;
@@ -164,8 +168,10 @@ int run(const char *name, int M, int N, int K, int L, bool a_rowmajor) {
 int main() {
   using GRow = FastGemm<cutlass::layout::RowMajor, cutlass::layout::ColumnMajor>;   // W = Vc^T B (A K-major)
   using GCol = FastGemm<cutlass::layout::ColumnMajor, cutlass::layout::ColumnMajor>; // C -= V W' (A M-major)
+  using GCol2 = FastGemm<cutlass::layout::ColumnMajor, cutlass::layout::ColumnMajor, true>;
   run<GRow>("W=VhC_256x96x160", 96, 160, 256, 2368, true);
   run<GCol>("C-=VW_256x160x96", 256, 160, 96, 2368, false);
+  run<GCol2>("C-=VW_256x160x96_2sm", 256, 160, 96, 2368, false);
   run<GRow>("W=VhC_192x96x96", 96, 96, 192, 2368, true);
   run<GCol>("C-=VW_192x96x96", 192, 96, 96, 2368, false);
   return 0;
