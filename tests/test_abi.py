@@ -219,3 +219,21 @@ def test_gauss_jordan_argument_checks(lib, args, code):
     d, n, nrhs, b, A, lda, B, ldb = args
     st = lib.bqr_gauss_jordan_batched(d, n, nrhs, b, ctypes.c_void_p(A), lda, ctypes.c_void_p(B), ldb, None, None)
     assert st == code
+
+
+def test_sass_proves_blackwell_native_instructions(lib):
+    """libbqr.so is built for sm_100a and its SASS contains the instructions
+    the design claims (B200_PROFILING.md "What proves a Blackwell-native
+    kernel"): tcgen05 MMA (UTCHMMA, the compact-WY tensor-core GEMMs), TMA
+    (UBLKCP bulk copies of the register-file kernels, UTMALDG in the GEMMs),
+    packed FP32 (FFMA2), and no legacy HMMA."""
+    import shutil
+    import subprocess
+    exe = shutil.which("cuobjdump") or "/usr/local/cuda/bin/cuobjdump"
+    if not os.path.exists(exe):
+        pytest.skip("cuobjdump not available")
+    out = subprocess.run([exe, "-sass", bqr._LIB_PATH], capture_output=True, text=True, timeout=600).stdout
+    assert "sm_100a" in subprocess.run([exe, "-lelf", bqr._LIB_PATH], capture_output=True, text=True).stdout
+    for mnem in ("UTCHMMA", "UBLKCP", "UTMALDG", "FFMA2"):
+        assert mnem in out, mnem
+    assert " HMMA" not in out
