@@ -527,7 +527,24 @@ int bqr_orgqr_batched(bqr_dtype_t dtype, int m, int n, int k, int batch, void *A
   if ((reinterpret_cast<uintptr_t>(A) | reinterpret_cast<uintptr_t>(tau)) % elem_size(dtype))
     return BQR_ERR_MISALIGNED;
   Plan p;
-  if (!orgqr_plan(dtype, m, n, &p)) return BQR_ERR_NOT_SUPPORTED;
+  if (!orgqr_plan(dtype, m, n, &p)) {
+    // beyond the single-SM classes (complex > 160): xORGQR by 96-column
+    // compact-WY panels on the tensor cores, workspace from the private pool
+    if (!wy_supported(dtype, m, n, lda) || (reinterpret_cast<uintptr_t>(A) & 15))
+      return BQR_ERR_NOT_SUPPORTED;
+    const size_t per = orgqr_wy_workspace_bytes(dtype, m, n, k, 1);
+    const long long chunk = std::max<long long>(1, std::min<long long>(batch, (long long)(kWyMaxWorkspace / per)));
+    const size_t bytes = orgqr_wy_workspace_bytes(dtype, m, n, k, (int)chunk);
+    cudaMemPool_t pool = wy_pool();
+    void *ws = nullptr;
+    if (!pool || cudaMallocFromPoolAsync(&ws, bytes, pool, stream) != cudaSuccess) {
+      cudaGetLastError();
+      return BQR_ERR_CUDA;
+    }
+    const int st = orgqr_wy(dtype, m, n, k, batch, A, lda, tau, ws, bytes, stream);
+    cudaFreeAsync(ws, stream);
+    return st;
+  }
   Call c{A, const_cast<void *>(tau), batch, m, n, k, lda, stream};
   c.strideT = n;  // tau batch stride min(m, n) = n, as bqr_geqrf_batched wrote it
   return p.orgqr(c);

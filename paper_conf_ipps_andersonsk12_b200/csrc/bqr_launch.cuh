@@ -210,6 +210,9 @@ bool wy_supported(bqr_dtype_t dt, int m, int n, int lda);
 size_t wy_workspace_bytes(bqr_dtype_t dt, int m, int n, int chunk);
 int geqrf_wy(bqr_dtype_t dt, int m, int n, long long batch, void *A, int lda, void *tau, void *work, size_t work_bytes,
              cudaStream_t stream, const Plan *(*pick_panel)(int, int));
+size_t orgqr_wy_workspace_bytes(bqr_dtype_t dt, int m, int n, int k, int chunk);
+int orgqr_wy(bqr_dtype_t dt, int m, int n, int k, long long batch, void *A, int lda, const void *tau, void *work,
+             size_t work_bytes, cudaStream_t stream);
 // back substitution X = R^{-1} C of the least-squares path (bqr_solve.cu)
 int solve_upper_dispatch(bqr_dtype_t dt, const void *A, int lda, long long strideA, void *B, int ldb,
                          long long strideB, int *info, long long batch, int n, int nrhs, cudaStream_t s);

@@ -41,6 +41,10 @@ int geqrf_wy(bqr_dtype_t, int, int, long long, void *, int, void *, void *, size
              const Plan *(*)(int, int)) {
   return BQR_ERR_NOT_SUPPORTED;
 }
+size_t orgqr_wy_workspace_bytes(bqr_dtype_t, int, int, int, int) { return 0; }
+int orgqr_wy(bqr_dtype_t, int, int, int, long long, void *, int, const void *, void *, size_t, cudaStream_t) {
+  return BQR_ERR_NOT_SUPPORTED;
+}
 }  // namespace host
 }  // namespace bqr
 #else
@@ -123,7 +127,8 @@ struct Gemm {
 // V (m_p x nb, unit lower trapezoidal) of each matrix's panel and, for
 // complex data, conj(V) (the K-major A operand of V^H X)
 template <class E>
-__global__ void extract_v_kernel(const E *A, long long sA, int lda, int k0, int mp, int nb, long long L, E *V, E *Vc) {
+__global__ void extract_v_kernel(const E *A, long long sA, int lda, int k0, int mp, int nb, long long L, E *V, E *Vc,
+                                 int nvalid = 1 << 30) {
   using X = El<E>;
   const long long per = (long long)mp * nb;
   for (long long idx = blockIdx.x * (long long)blockDim.x + threadIdx.x; idx < per * L;
@@ -131,8 +136,8 @@ __global__ void extract_v_kernel(const E *A, long long sA, int lda, int k0, int 
     const long long b = idx / per;
     const int rem = (int)(idx - b * per);
     const int i = rem / mp, r = rem - i * mp;  // column i, row r
-    E v = r == i ? X::one() : X::zero();
-    if (r > i) v = A[b * sA + (long long)(k0 + i) * lda + (k0 + r)];
+    E v = r == i && i < nvalid ? X::one() : X::zero();  // columns >= nvalid: zero padding
+    if (r > i && i < nvalid) v = A[b * sA + (long long)(k0 + i) * lda + (k0 + r)];
     V[idx] = v;
     if constexpr (X::kComplex) Vc[idx] = X::conj(v);
   }
@@ -154,7 +159,8 @@ __device__ __forceinline__ void mac(float &s, float a, float b) { s = fmaf(a, b,
 // Writes Th = T^H (nb x nb, column-major).  One CTA per matrix.
 constexpr int kTB = 16;
 template <class E>
-__global__ void __launch_bounds__(256) larft_kernel(const E *G, const E *tau, long long sTau, int nb, E *Th) {
+__global__ void __launch_bounds__(256) larft_kernel(const E *G, const E *tau, long long sTau, int nb, E *Th,
+                                                    bool herm = true, int nvalid = 1 << 30) {
   using X = El<E>;
   extern __shared__ __align__(16) unsigned char tsm_raw[];
   E *T = reinterpret_cast<E *>(tsm_raw);  // nb x nb column-major, then P (nb x kTB)
@@ -171,7 +177,7 @@ __global__ void __launch_bounds__(256) larft_kernel(const E *G, const E *tau, lo
     const int j0 = d * kTB, bs = min(kTB, nb - j0);
     for (int ii = 0; ii < bs; ++ii) {
       const int i = j0 + ii;
-      const E ti = tb[i];
+      const E ti = i < nvalid ? tb[i] : X::zero();  // padded reflectors: tau = 0, H = I
       if (lane < ii) {
         E sum = X::zero();
         for (int l = j0 + lane; l < i; ++l) mac(sum, T[(j0 + lane) + l * nb], __ldg(Gb + l + i * nb));
@@ -204,8 +210,23 @@ __global__ void __launch_bounds__(256) larft_kernel(const E *G, const E *tau, lo
   }
   E *Thb = Th + b * (long long)nb * nb;
   for (int q = tid; q < nb * nb; q += blockDim.x) {
-    const int r = q % nb, c = q / nb;  // Th(r, c) = conj(T(c, r))
-    Thb[q] = X::conj(T[c + r * nb]);
+    const int r = q % nb, c = q / nb;  // Th(r, c) = conj(T(c, r)), or T itself (orgqr)
+    Thb[q] = herm ? X::conj(T[c + r * nb]) : T[q];
+  }
+}
+
+// the first n columns of the m x m identity (xORGQR's starting point);
+// padding rows lda > m untouched
+template <class E>
+__global__ void eye_kernel(E *A, long long sA, int lda, int m, int n, long long L) {
+  using X = El<E>;
+  const long long per = (long long)m * n;
+  for (long long idx = blockIdx.x * (long long)blockDim.x + threadIdx.x; idx < per * L;
+       idx += (long long)gridDim.x * blockDim.x) {
+    const long long b = idx / per;
+    const int rem = (int)(idx - b * per);
+    const int c = rem / m, r = rem - c * m;
+    A[b * sA + (long long)c * lda + r] = r == c ? X::one() : X::zero();
   }
 }
 
@@ -304,6 +325,108 @@ int geqrf_wy(bqr_dtype_t dt, int m, int n, long long batch, void *A, int lda, vo
              size_t work_bytes, cudaStream_t stream, const Plan *(*pick_panel)(int, int)) {
   return dt == BQR_R32 ? geqrf_wy_t<float>(m, n, batch, A, lda, tau, work, work_bytes, stream, pick_panel)
                        : geqrf_wy_t<float2>(m, n, batch, A, lda, tau, work, work_bytes, stream, pick_panel);
+}
+
+// ---- xORGQR by panels (bqr_orgqr_batched beyond the single-SM classes):
+// Q = Q_0 Q_1 ... Q_{p-1}, Q_j = I - V_j T_j V_j^H; starting from the first n
+// columns of I, Q_j is applied backwards to rows / columns k0_j.. (the
+// columns left of k0_j are still unit vectors that V_j^H maps to 0).
+static size_t orgqr_wy_bytes_per_matrix(bqr_dtype_t dt, int m, int n, int k) {
+  const size_t es = dt == BQR_R32 ? 4 : 8;
+  const int nb = wy_panel_width(dt);
+  size_t v = 0, t = 0;
+  for (int k0 = 0; k0 < k; k0 += nb) {
+    const int w = std::min(nb, (k - k0 + 3) & ~3);
+    v += (size_t)(m - k0) * w;
+    t += (size_t)w * w;
+  }
+  return es * ((dt == BQR_R32 ? 1 : 2) * v + t + (size_t)nb * nb + 2 * (size_t)nb * n) + 256;
+}
+
+size_t orgqr_wy_workspace_bytes(bqr_dtype_t dt, int m, int n, int k, int chunk) {
+  return chunk * orgqr_wy_bytes_per_matrix(dt, m, n, k) + 1024;
+}
+
+template <class E>
+static int orgqr_wy_t(int m, int n, int k, long long batch, void *A, int lda, const void *tau, void *work,
+                      size_t work_bytes, cudaStream_t stream) {
+  using T = wy::Tr<E>;
+  constexpr bool kC = El<E>::kComplex;
+  const bqr_dtype_t dt = kC ? BQR_C64 : BQR_R32;
+  const int nb = wy_panel_width(dt);
+  const long long sA = (long long)lda * n;
+  const size_t per = orgqr_wy_bytes_per_matrix(dt, m, n, k);
+  long long chunk = (long long)(work_bytes / per);
+  if (chunk < 1) return -10;
+  chunk = std::min(chunk, batch);
+  using GRow = wy::Gemm<E, cutlass::layout::RowMajor>;
+  using GCol = wy::Gemm<E, cutlass::layout::ColumnMajor>;
+  const int np = (k + nb - 1) / nb;
+  // panel widths padded to the TMA's 16-byte row alignment with zero
+  // reflectors (tau = 0, H = I): an odd last panel keeps the GEMM operands aligned
+  const int al = kC ? 2 : 4;
+  auto width = [&](int k0) { return std::min(nb, (k - k0 + al - 1) / al * al); };
+  for (long long b0 = 0; b0 < batch; b0 += chunk) {
+    const long long L = std::min(chunk, batch - b0);
+    E *Ab = reinterpret_cast<E *>(A) + b0 * sA;
+    const E *tb = reinterpret_cast<const E *>(tau) + b0 * n;
+    E *ws = reinterpret_cast<E *>((reinterpret_cast<uintptr_t>(work) + 255) & ~uintptr_t(255));
+    // carve: per panel V_j, Vc_j (L x (m - k0) x w) and T_j (L x w x w); G; W; X
+    E *Vp[16], *Vcp[16], *Tp[16];
+    if (np > 16) return BQR_ERR_NOT_SUPPORTED;
+    E *cur = ws;
+    for (int j = 0; j < np; ++j) {
+      const int k0 = j * nb, w = width(k0), mj = m - k0;
+      Vp[j] = cur;
+      cur += (size_t)L * mj * w;
+      Vcp[j] = kC ? cur : Vp[j];
+      if (kC) cur += (size_t)L * mj * w;
+      Tp[j] = cur;
+      cur += (size_t)L * w * w;
+    }
+    E *G = cur;
+    E *W = G + (size_t)L * nb * nb;
+    E *X = W + (size_t)L * nb * n;
+    // 1. V_j and T_j of every panel while A still holds the reflectors
+    for (int j = 0; j < np; ++j) {
+      const int k0 = j * nb, w = width(k0), mj = m - k0;
+      const long long nv = (long long)L * mj * w;
+      wy::extract_v_kernel<E><<<(unsigned)std::min<long long>((nv + 255) / 256, 148 * 64), 256, 0, stream>>>(
+          Ab, sA, lda, k0, mj, w, L, Vp[j], Vcp[j], k - k0);
+      if (cudaGetLastError() != cudaSuccess) return BQR_ERR_CUDA;
+      const int64_t sV = (int64_t)mj * w, sG = (int64_t)w * w;
+      int st = GRow::run(w, w, mj, (int)L, Vcp[j], mj, sV, Vp[j], mj, sV, G, w, sG, T::one(), T::zero(), stream);
+      if (st != BQR_SUCCESS) return st;
+      const size_t tsm = (size_t)(w * w + w * wy::kTB) * sizeof(E);
+      if (!ensure_smem(reinterpret_cast<const void *>(wy::larft_kernel<E>), tsm)) return BQR_ERR_CUDA;
+      wy::larft_kernel<E><<<(unsigned)L, 256, tsm, stream>>>(G, tb + k0, n, w, Tp[j], false, k - k0);
+      if (cudaGetLastError() != cudaSuccess) return BQR_ERR_CUDA;
+    }
+    // 2. A <- I (m x n)
+    const long long ne = (long long)L * m * n;
+    wy::eye_kernel<E><<<(unsigned)std::min<long long>((ne + 255) / 256, 148 * 64), 256, 0, stream>>>(Ab, sA, lda, m,
+                                                                                                       n, L);
+    if (cudaGetLastError() != cudaSuccess) return BQR_ERR_CUDA;
+    // 3. E[k0:m, k0:n] <- Q_j E[k0:m, k0:n], j = p-1 .. 0
+    for (int j = np - 1; j >= 0; --j) {
+      const int k0 = j * nb, w = width(k0), mj = m - k0, nc = n - k0;
+      const int64_t sV = (int64_t)mj * w, sG = (int64_t)w * w, sW = (int64_t)w * nc;
+      E *Eb = Ab + k0 + (size_t)k0 * lda;
+      int st = GRow::run(w, nc, mj, (int)L, Vcp[j], mj, sV, Eb, lda, sA, W, w, sW, T::one(), T::zero(), stream);
+      if (st != BQR_SUCCESS) return st;
+      st = GCol::run(w, nc, w, (int)L, Tp[j], w, sG, W, w, sW, X, w, sW, T::one(), T::zero(), stream);
+      if (st != BQR_SUCCESS) return st;
+      st = GCol::run(mj, nc, w, (int)L, Vp[j], mj, sV, X, w, sW, Eb, lda, sA, T::mone(), T::one(), stream);
+      if (st != BQR_SUCCESS) return st;
+    }
+  }
+  return BQR_SUCCESS;
+}
+
+int orgqr_wy(bqr_dtype_t dt, int m, int n, int k, long long batch, void *A, int lda, const void *tau, void *work,
+             size_t work_bytes, cudaStream_t stream) {
+  return dt == BQR_R32 ? orgqr_wy_t<float>(m, n, k, batch, A, lda, tau, work, work_bytes, stream)
+                       : orgqr_wy_t<float2>(m, n, k, batch, A, lda, tau, work, work_bytes, stream);
 }
 
 }  // namespace host
