@@ -414,13 +414,14 @@ int bqr_geqrf_launches(bqr_dtype_t dtype, int m, int n, int batch) {
   const bool wy = wy_default_shape(dtype, m, n, m);
   const int kmax = std::min(m, n);
   // per panel: tiled = panel + apply; WY = panel + V extraction + 4 GEMMs + xLARFT
+  // + the accumulate C += D
   // (one chunk when the batch fits the default path's workspace)
   const long long per_chunk =
       wy ? std::max<long long>(1, (long long)(kWyMaxWorkspace / wy_workspace_bytes(dtype, m, n, 1))) : batch;
   const long long chunks = (batch + per_chunk - 1) / per_chunk;
   int launches = 0;
   for (int k0 = 0; k0 < kmax; k0 += nb)
-    launches += (n - k0 - std::min(nb, kmax - k0) > 0) ? (wy ? 7 : 2) : 1;
+    launches += (n - k0 - std::min(nb, kmax - k0) > 0) ? (wy ? 8 : 2) : 1;
   return (int)(launches * chunks);
 }
 

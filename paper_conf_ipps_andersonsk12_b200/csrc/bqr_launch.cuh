@@ -3,6 +3,7 @@
 // parallel): the per-call descriptor, the plan table entry, and the
 // launch templates of the register-file, tiny and Q^H B kernels.
 #pragma once
+#include <cstdlib>
 #include <cuda_runtime.h>
 
 #include <algorithm>
@@ -117,6 +118,11 @@ int launch_rf(const Call &c) {
     int sms = 0, bps = 0;
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, current_device());
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, kern, Cfg::NT, smem);
+    static const int cap = [] {  // experiment knob: resident CTAs per SM
+      const char *e = std::getenv("BQR_MAX_BPS");
+      return e ? std::atoi(e) : 0;
+    }();
+    if (cap > 0) bps = std::min(bps, cap);
     grid = std::min<long long>(grid, std::max(1, sms * std::max(1, bps)));
   }
   if (grid > 0x7fffffffLL) return BQR_ERR_NOT_SUPPORTED;

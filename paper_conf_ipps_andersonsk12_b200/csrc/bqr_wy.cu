@@ -215,6 +215,29 @@ __global__ void __launch_bounds__(256) larft_kernel(const E *G, const E *tau, lo
   }
 }
 
+// C += D over the trailing block (C: ld ldc, batch stride sC; D: dense
+// mp x nt, ld mp): the accumulate of the update C - V X, kept out of the
+// GEMM epilogue (CUTLASS's transform epilogue reads a complex source 4x
+// slower than the whole beta = 0 GEMM, profiles/r02/experiments)
+template <class E>
+__global__ void add_block_kernel(E *C, int ldc, long long sC, const E *D, int mp, int nt, long long L) {
+  const long long per = (long long)mp * nt;
+  for (long long idx = blockIdx.x * (long long)blockDim.x + threadIdx.x; idx < per * L;
+       idx += (long long)gridDim.x * blockDim.x) {
+    const long long b = idx / per;
+    const int rem = (int)(idx - b * per);
+    const int j = rem / mp, i = rem - j * mp;
+    E &c = C[b * sC + (long long)j * ldc + i];
+    const E d = D[idx];
+    if constexpr (El<E>::kComplex) {
+      c.x += d.x;
+      c.y += d.y;
+    } else {
+      c += d;
+    }
+  }
+}
+
 // the first n columns of the m x m identity (xORGQR's starting point);
 // padding rows lda > m untouched
 template <class E>
@@ -241,7 +264,10 @@ int wy_panel_width(bqr_dtype_t dt) { return dt == BQR_R32 ? 64 : 96; }
 static size_t wy_bytes_per_matrix(bqr_dtype_t dt, int m, int n, int nb) {
   const size_t es = dt == BQR_R32 ? 4 : 8;
   const size_t V = (size_t)m * nb, G = (size_t)nb * nb, W = (size_t)nb * std::max(0, n - nb);
-  return es * ((dt == BQR_R32 ? 1 : 2) * V + 2 * G + 2 * W) + 256;
+  // V X before the accumulate: complex data reuse the dead conj(V), G, T^H
+  // and W (m <= 256: m_p n_t <= m_p nb + 2 nb^2 + nb n_t), real data need it
+  const size_t D = dt == BQR_R32 ? (size_t)m * std::max(0, n - nb) : 0;
+  return es * ((dt == BQR_R32 ? 1 : 2) * V + 2 * G + 2 * W + D) + 256;
 }
 
 // shapes the blocked variant can take: the TMA rows of V, C and W need
@@ -255,6 +281,14 @@ bool wy_supported(bqr_dtype_t dt, int m, int n, int lda) {
 
 size_t wy_workspace_bytes(bqr_dtype_t dt, int m, int n, int chunk) {
   return chunk * wy_bytes_per_matrix(dt, m, n, wy_panel_width(dt)) + 1024;
+}
+
+template <class E>
+static int add_block(E *C, int ldc, long long sC, const E *D, int mp, int nt, long long L, cudaStream_t stream) {
+  const long long ne = (long long)L * mp * nt;
+  wy::add_block_kernel<E><<<(unsigned)std::min<long long>((ne + 255) / 256, 148 * 64), 256, 0, stream>>>(
+      C, ldc, sC, D, mp, nt, L);
+  return cudaGetLastError() == cudaSuccess ? BQR_SUCCESS : BQR_ERR_CUDA;
 }
 
 template <class E>
@@ -294,6 +328,7 @@ static int geqrf_wy_t(int m, int n, long long batch, void *A, int lda, void *tau
       E *Th = G + (size_t)L * w * w;
       E *W = Th + (size_t)L * w * w;
       E *X = W + (size_t)L * w * nt;
+      E *Dw = kC ? Vc : X + (size_t)L * w * nt;  // Vc .. W are dead once X is formed
       const long long nv = (long long)L * mp * w;
       wy::extract_v_kernel<E><<<(unsigned)std::min<long long>((nv + 255) / 256, 148 * 64), 256, 0, stream>>>(
           Ab, sA, lda, k0, mp, w, L, V, Vc);
@@ -313,8 +348,11 @@ static int geqrf_wy_t(int m, int n, long long batch, void *A, int lda, void *tau
       // X = T^H W
       st = GCol::run(w, nt, w, (int)L, Th, w, sG, W, w, sW, X, w, sW, T::one(), T::zero(), stream);
       if (st != BQR_SUCCESS) return st;
-      // C = C - V X
-      st = GCol::run(mp, nt, w, (int)L, V, mp, sV, X, w, sW, Cb, lda, sA, T::mone(), T::one(), stream);
+      // C = C - V X: D = -V X (beta = 0), then C += D
+      const int64_t sD = (int64_t)mp * nt;
+      st = GCol::run(mp, nt, w, (int)L, V, mp, sV, X, w, sW, Dw, mp, sD, T::mone(), T::zero(), stream);
+      if (st != BQR_SUCCESS) return st;
+      st = add_block(Cb, lda, sA, Dw, mp, nt, L, stream);
       if (st != BQR_SUCCESS) return st;
     }
   }
@@ -340,7 +378,7 @@ static size_t orgqr_wy_bytes_per_matrix(bqr_dtype_t dt, int m, int n, int k) {
     v += (size_t)(m - k0) * w;
     t += (size_t)w * w;
   }
-  return es * ((dt == BQR_R32 ? 1 : 2) * v + t + (size_t)nb * nb + 2 * (size_t)nb * n) + 256;
+  return es * ((dt == BQR_R32 ? 1 : 2) * v + t + (size_t)nb * nb + 2 * (size_t)nb * n + (size_t)m * n) + 256;
 }
 
 size_t orgqr_wy_workspace_bytes(bqr_dtype_t dt, int m, int n, int k, int chunk) {
@@ -387,6 +425,7 @@ static int orgqr_wy_t(int m, int n, int k, long long batch, void *A, int lda, co
     E *G = cur;
     E *W = G + (size_t)L * nb * nb;
     E *X = W + (size_t)L * nb * n;
+    E *Dw = X + (size_t)L * nb * n;
     // 1. V_j and T_j of every panel while A still holds the reflectors
     for (int j = 0; j < np; ++j) {
       const int k0 = j * nb, w = width(k0), mj = m - k0;
@@ -416,7 +455,10 @@ static int orgqr_wy_t(int m, int n, int k, long long batch, void *A, int lda, co
       if (st != BQR_SUCCESS) return st;
       st = GCol::run(w, nc, w, (int)L, Tp[j], w, sG, W, w, sW, X, w, sW, T::one(), T::zero(), stream);
       if (st != BQR_SUCCESS) return st;
-      st = GCol::run(mj, nc, w, (int)L, Vp[j], mj, sV, X, w, sW, Eb, lda, sA, T::mone(), T::one(), stream);
+      st = GCol::run(mj, nc, w, (int)L, Vp[j], mj, sV, X, w, sW, Dw, mj, (int64_t)mj * nc, T::mone(), T::zero(),
+                     stream);
+      if (st != BQR_SUCCESS) return st;
+      st = add_block(Eb, lda, sA, Dw, mj, nc, L, stream);
       if (st != BQR_SUCCESS) return st;
     }
   }
