@@ -2,6 +2,7 @@
 from __future__ import annotations
 
 import os
+import re
 import subprocess
 import sys
 
@@ -46,8 +47,22 @@ def stale() -> bool:
     return any(os.path.getmtime(s) > t for s in sources())
 
 
+def deps(path, seen=None):
+    """The translation unit and every quoted #include it reaches."""
+    seen = set() if seen is None else seen
+    if path in seen or not os.path.exists(path):
+        return seen
+    seen.add(path)
+    with open(path) as f:
+        for inc in re.findall(r'^\s*#\s*include\s+"([^"]+)"', f.read(), re.M):
+            deps(os.path.normpath(os.path.join(os.path.dirname(path), inc)), seen)
+    return seen
+
+
 def build(force: bool = False, verbose: bool = False, extra=()) -> str:
-    """Compile every csrc/*.cu translation unit in parallel, link libbqr.so."""
+    """Compile the csrc/*.cu translation units whose object is older than the
+    unit or a header it includes (all of them with force / extra flags) in
+    parallel, link libbqr.so."""
     if not force and not stale():
         return LIB
     units = sorted(f for f in os.listdir(CSRC) if f.endswith(".cu"))
@@ -57,6 +72,11 @@ def build(force: bool = False, verbose: bool = False, extra=()) -> str:
     procs = []
     for u in units:
         obj = os.path.join(objdir, u[:-3] + ".o")
+        src = os.path.join(CSRC, u)
+        if (not force and not extra and os.path.exists(obj)
+                and all(os.path.getmtime(d) <= os.path.getmtime(obj) for d in deps(src))):
+            procs.append((u, obj, None))
+            continue
         cmd = [NVCC, *cflags, *(cutlass_flags() if u == "bqr_wy.cu" else []), *extra, "-c", "-o", obj,
                os.path.join(CSRC, u)]
         if verbose:
@@ -65,7 +85,7 @@ def build(force: bool = False, verbose: bool = False, extra=()) -> str:
         procs.append((u, obj, subprocess.Popen(cmd)))
     objs = []
     for u, obj, pr in procs:
-        if pr.wait() != 0:
+        if pr is not None and pr.wait() != 0:
             raise subprocess.CalledProcessError(pr.returncode, f"nvcc {u}")
         objs.append(obj)
     link = [NVCC, "-shared", "-gencode", "arch=compute_100a,code=sm_100a", "-Xcompiler", "-fPIC",

@@ -61,15 +61,16 @@ using namespace bqr::host;
 // classes, then fp32, then complex64, then the
 // experiment-only alternatives (BQR_FORCE_VARIANT).
 struct Tables {
-  static constexpr int kN = 5;
+  static constexpr int kN = 6;
   const ClassEntry *t[kN];
   int n[kN];
   Tables() {
-    t[0] = classes_co(&n[0]);
-    t[1] = classes_headline(&n[1]);
-    t[2] = classes_f32(&n[2]);
-    t[3] = classes_c64(&n[3]);
-    t[4] = classes_alt(&n[4]);
+    t[0] = classes_ll(&n[0]);
+    t[1] = classes_co(&n[1]);
+    t[2] = classes_headline(&n[2]);
+    t[3] = classes_f32(&n[3]);
+    t[4] = classes_c64(&n[4]);
+    t[5] = classes_alt(&n[5]);
   }
   template <class F>
   const Plan *find(F pred) const {

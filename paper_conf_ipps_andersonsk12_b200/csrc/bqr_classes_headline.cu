@@ -9,7 +9,9 @@ namespace host {
 
 namespace {
 const ClassEntry kTable[] = {
-    {BQR_R32, 56, 56, 56, 56, false, RF_PLAN_X(float, 4, 4, 14, 14, 2, true, true, "rf_f32_R4G4_14x14_x2_exact")},
+    // the round-1/2 right-looking C3 class; the dispatched one is the
+    // left-looking bqr_classes_ll.cu (A/B via BQR_FORCE_VARIANT)
+    {BQR_R32, 56, 56, 56, 56, true, RF_PLAN_X(float, 4, 4, 14, 14, 2, true, true, "alt_rf_f32_R4G4_14x14_x2_exact")},
     {BQR_C64, 240, 66, 240, 66, false, RF_PLAN(float2, 32, 11, 8, 6, 1, false, "rf_c64_R32G11_8x6_cta")},
     // NEXT-2: the paper's other RT_STAP shapes (Table VII)
     {BQR_C64, 80, 16, 80, 16, false, RF_PLAN(float2, 16, 4, 5, 4, 1, false, "rf_c64_R16G4_5x4_cta")},

@@ -1,0 +1,333 @@
+// bqr_ll.cuh -- left-looking register-block Householder QR for the C3
+// headline shape (56 x 56 fp32; BASELINE config 3, "5,000
+// 56x56 QR factorizations").
+//
+// Same arithmetic as the right-looking register-file classes (bqr_rf.cuh):
+// xLARFG per column (norm, IEEE sqrt/div: "a square root, two divides, and
+// two multiplies") and H_k = I - tau_k v_k v_k^T applied as a
+// matrix-vector product plus a rank-1 update (Table VI), in the
+// paper's 2D-cyclic register layout (Fig. 6) with 4 row lanes x
+// 4 column groups per matrix, two matrices per warp.  What changes is the
+// ORDER of the column updates (a "blocked algorithm"):
+//
+//   * the 56 columns are factored in three column blocks [0,20) [20,36)
+//     [36,56); only the current block lives in registers (<= 14 rows x 5
+//     slots per lane instead of the whole 14 x 14 tile), so the kernel holds
+//     17 warps = 34 matrices per SM at <= 120 registers: 5,000 matrices are
+//     ONE resident round on 148 SMs (the right-looking class holds 16 per SM
+//     at 255 registers: 2.11 rounds, 2 warps per scheduler, IPC 1.6);
+//   * a block is loaded from HBM when it is reached, H_0..H_{c0-1} of the
+//     earlier blocks are applied to it (left-looking: the reflectors are
+//     known, so this is pure matrix-vector/rank-1 throughput with no
+//     reflector chain), then it is factored right-looking with a one-column
+//     look-ahead (apply H_k to the slot of column k+1, form reflector k+1,
+//     apply H_k to the other slots) and written back;
+//   * the Householder vectors of the first two blocks stay in shared memory
+//     (row-lane-major, rows from the reflector's first live register-row
+//     pair, 6.3 KB per matrix) for the later blocks; the last block
+//     publishes through a two-entry ring;
+//   * packed FP32 (fma.rn.f32x2, SASS FFMA2) on register-row pairs
+//     (rows rg + 8p, rg + 8p + 4): v pairs come straight from 8-byte shared
+//     loads, so no operand moves are needed.
+// Rows of a reflector above its pivot are stored as exact zeros, so the
+// applies need no row masks; only the pivot's register row is masked in the
+// reflector itself and the pivot slot's columns <= k in the update.
+#pragma once
+#include "bqr_common.cuh"
+
+namespace bqr {
+namespace ll {
+
+struct LlArgs {
+  float *A;
+  float *tau;
+  long long batch;
+  int lda;
+  long long strideA, strideT;
+};
+
+constexpr int kM = 56;      // rows = columns
+constexpr int MP = 7;       // register-row pairs per lane: rows rg + 8p, rg + 8p + 4
+constexpr int NSMAX = 4;    // column slots per lane of a block (columns c0 + cg + 4j)
+constexpr int kWarps = 17;  // one CTA of 17 warps (34 matrices) per SM
+constexpr int kThreads = 32 * kWarps;
+// column blocks [0,16) [16,28) [28,40) [40,56)
+__host__ __device__ constexpr int blk_c0(int b) { return b == 0 ? 0 : (b == 1 ? 16 : (b == 2 ? 28 : 40)); }
+__host__ __device__ constexpr int blk_ns(int b) { return b == 0 ? 4 : (b == 1 ? 3 : (b == 2 ? 3 : 4)); }
+constexpr int kNB = 4;
+// reflectors of panels 0..9 (columns 0..39) are kept for the left-looking
+// applies; panel P's vector holds this lane's pairs P/2 .. MP-1
+constexpr int kKeepP = 10;
+__host__ __device__ constexpr int vlen(int P) { return 2 * (MP - P / 2); }
+__host__ __device__ constexpr int voff(int P) { return P == 0 ? 0 : voff(P - 1) + 16 * vlen(P - 1); }
+constexpr int kVStore = voff(kKeepP);       // 1600 words
+constexpr int kRingQ = kKeepP / 2;          // first pair of the ring vectors
+constexpr int kRingOff = kVStore;           // 2 x [4 row lanes][pairs kRingQ..6]
+constexpr int kRingLen = 2 * (MP - kRingQ);
+constexpr int kRingBuf = 4 * kRingLen;
+constexpr int kTauOff = kRingOff + 2 * kRingBuf;
+constexpr int kMatWords = kTauOff + kM;     // 1688 words: 34 matrices = 224 KB
+constexpr size_t kSmemBytes = (size_t)kWarps * 2 * kMatWords * 4;
+static_assert(NSMAX == 4, "do_block loads slots 0..3");
+static_assert(kMatWords % 2 == 0, "8-byte aligned vectors");
+static_assert(kSmemBytes <= 232448, "one CTA of 34 matrices per SM");
+static_assert(blk_c0(kNB - 1) == 4 * kKeepP && blk_c0(kNB - 1) + 4 * blk_ns(kNB - 1) == kM, "blocks");
+
+__device__ __forceinline__ void wsync() { asm volatile("bar.warp.sync -1;" ::: "memory"); }
+__device__ __forceinline__ float2 lds64(const float *p) {
+  float2 v;
+  const unsigned s = (unsigned)__cvta_generic_to_shared(p);
+  asm volatile("ld.shared.v2.f32 {%0,%1}, [%2];" : "=f"(v.x), "=f"(v.y) : "r"(s));
+  return v;
+}
+__device__ __forceinline__ void sts64(float *p, float2 v) {
+  const unsigned s = (unsigned)__cvta_generic_to_shared(p);
+  asm volatile("st.shared.v2.f32 [%0], {%1,%2};" ::"r"(s), "f"(v.x), "f"(v.y) : "memory");
+}
+
+struct Ctx {
+  float *sm;    // this matrix's shared words
+  float *Ab;    // this lane's element (rg, cg) of the matrix in global memory
+  int lda;
+  int rg, cg, lane;
+};
+
+// this lane's vector of reflector k = 4P + kk, positioned at pair P/2
+template <int P>
+__device__ __forceinline__ float *vptr(const Ctx &c, int kk) {
+  if constexpr (P < kKeepP) {
+    return c.sm + voff(P) + (kk * 4 + c.rg) * vlen(P);
+  } else {
+    return c.sm + kRingOff + (kk & 1) * kRingBuf + c.rg * kRingLen + (P / 2 - kRingQ) * 2;
+  }
+}
+
+using Tile = float2[MP][NSMAX];
+
+// slot j of block B (columns c0 + cg + 4j, rows rg + 4i) <-> HBM
+template <int B, int J>
+__device__ __forceinline__ void load_slot(const Ctx &c, Tile &a) {
+  if constexpr (B < kNB && J < blk_ns(B)) {
+    const float *col = c.Ab + (long long)(blk_c0(B) + 4 * J) * c.lda;
+#pragma unroll
+    for (int p = 0; p < MP; ++p) a[p][J] = make_float2(col[8 * p], col[8 * p + 4]);
+  }
+}
+template <int B, int J>
+__device__ __forceinline__ void store_slot(const Ctx &c, const Tile &a) {
+  float *col = c.Ab + (long long)(blk_c0(B) + 4 * J) * c.lda;
+#pragma unroll
+  for (int p = 0; p < MP; ++p) {
+    col[8 * p] = a[p][J].x;
+    col[8 * p + 4] = a[p][J].y;
+  }
+}
+
+
+// H_k = I - tau v v^T on slots [J0, J1), rows from pair Q0 (v is zero above
+// its pivot); MASK0: slot J0 only for the columns cg > kk (pivot slot)
+template <int Q0, int J0, int J1, bool MASK0>
+__device__ __forceinline__ void apply(const Ctx &c, Tile &a, const float *vp, float tau, int kk) {
+  if constexpr (J0 < J1) {
+    constexpr int NS = J1 - J0;
+    float2 v[MP];
+#pragma unroll
+    for (int p = Q0; p < MP; ++p) v[p] = lds64(vp + 2 * (p - Q0));
+    float2 w[NS];
+#pragma unroll
+    for (int j = 0; j < NS; ++j) w[j] = make_float2(0.f, 0.f);
+#pragma unroll
+    for (int p = Q0; p < MP; ++p)
+#pragma unroll
+      for (int j = 0; j < NS; ++j) w[j] = __ffma2_rn(v[p], a[p][J0 + j], w[j]);
+    float s[NS];
+#pragma unroll
+    for (int j = 0; j < NS; ++j) s[j] = w[j].x + w[j].y;
+#pragma unroll
+    for (int j = 0; j < NS; ++j) s[j] += __shfl_xor_sync(0xffffffffu, s[j], 1);
+#pragma unroll
+    for (int j = 0; j < NS; ++j) s[j] += __shfl_xor_sync(0xffffffffu, s[j], 2);
+    float2 nt[NS];
+#pragma unroll
+    for (int j = 0; j < NS; ++j) {
+      float t = tau * s[j];
+      if (MASK0 && j == 0) t = c.cg > kk ? t : 0.f;
+      nt[j] = make_float2(-t, -t);
+    }
+#ifdef BQR_LL_RELOAD
+#pragma unroll
+    for (int p = Q0; p < MP; ++p) v[p] = lds64(vp + 2 * (p - Q0));
+#endif
+#pragma unroll
+    for (int p = Q0; p < MP; ++p)
+#pragma unroll
+      for (int j = 0; j < NS; ++j) a[p][J0 + j] = __ffma2_rn(v[p], nt[j], a[p][J0 + j]);
+  }
+}
+
+// xLARFG of column kn = 4 PP + kkn held in slot S (computed by every lane;
+// the owner column group cg == kkn uses it)
+template <int PP, int S>
+__device__ __forceinline__ Reflector<float> reflector(const Ctx &c, const Tile &a, int kkn) {
+  constexpr int q0 = PP / 2;
+  float2 acc[2] = {make_float2(0.f, 0.f), make_float2(0.f, 0.f)};
+  float alpha = 0.f;
+#pragma unroll
+  for (int p = q0; p < MP; ++p) {
+    float2 x = a[p][S];
+    if (p == q0) {
+      if constexpr (PP % 2 == 0) {
+        alpha = c.rg == kkn ? x.x : 0.f;
+        x.x = c.rg > kkn ? x.x : 0.f;
+      } else {
+        alpha = c.rg == kkn ? x.y : 0.f;
+        x.y = c.rg > kkn ? x.y : 0.f;
+        x.x = 0.f;
+      }
+    }
+    acc[(p - q0) & 1] = __ffma2_rn(x, x, acc[(p - q0) & 1]);
+  }
+  const float2 accs = __fadd2_rn(acc[0], acc[1]);
+  float sig = accs.x + accs.y;
+  sig += __shfl_xor_sync(0xffffffffu, sig, 1);
+  sig += __shfl_xor_sync(0xffffffffu, sig, 2);
+  alpha = __shfl_sync(0xffffffffu, alpha, (c.lane & ~3) | kkn);
+  return make_reflector(alpha, sig);
+}
+
+// owner lanes: v = x * scal below the pivot, 1 at it, 0 above; the column
+// becomes [R; V] (beta at the pivot); v and tau go to shared memory.
+// Non-owner lanes multiply by 1 (bit-exact no-op), branch-free.
+template <int PP, int S>
+__device__ __forceinline__ void publish(const Ctx &c, Tile &a, const Reflector<float> &h, int kkn, float *vdst,
+                                        float *tslot) {
+  constexpr int q0 = PP / 2;
+  const bool own = c.cg == kkn;
+  const float scal = own ? h.scal : 1.f;
+#pragma unroll
+  for (int p = q0; p < MP; ++p) {
+    const float2 x = a[p][S];
+    const float2 xs = make_float2(x.x * scal, x.y * scal);
+    float2 v = xs, nx = xs;
+    if (p == q0) {
+      if constexpr (PP % 2 == 0) {
+        v.x = c.rg > kkn ? xs.x : (c.rg == kkn ? 1.f : 0.f);
+        nx.x = c.rg > kkn ? xs.x : ((own && c.rg == kkn) ? h.beta : x.x);
+      } else {
+        v.x = 0.f;
+        nx.x = x.x;
+        v.y = c.rg > kkn ? xs.y : (c.rg == kkn ? 1.f : 0.f);
+        nx.y = c.rg > kkn ? xs.y : ((own && c.rg == kkn) ? h.beta : x.y);
+      }
+    }
+    a[p][S] = nx;
+    if (own) *reinterpret_cast<float2 *>(vdst + 2 * (p - q0)) = v;
+  }
+  if (own && c.rg == 0) *tslot = h.tau;
+}
+
+// ---------------------------------------------------------------- phases
+// left-looking: H_0 .. H_{c0-1} (panels 0 .. c0/4 - 1) on block B
+template <int B, int P>
+__device__ __forceinline__ void left(const Ctx &c, Tile &a) {
+  if constexpr (P < blk_c0(B) / 4) {
+    const float *taus = c.sm + kTauOff;
+#pragma unroll 1
+    for (int kk = 0; kk < 4; ++kk) apply<P / 2, 0, blk_ns(B), false>(c, a, vptr<P>(c, kk), taus[4 * P + kk], kk);
+    left<B, P + 1>(c, a);
+  }
+}
+
+// right-looking factorisation of block B, panel P (slot s = P - c0/4), with
+// the one-column look-ahead; reflector 4P is published on entry
+template <int B, int P>
+__device__ __forceinline__ void panels(const Ctx &c, Tile &a) {
+  constexpr int P0 = blk_c0(B) / 4, NS = blk_ns(B);
+  if constexpr (P < P0 + NS) {
+    constexpr int s = P - P0, q0 = P / 2;
+    float *taus = c.sm + kTauOff;
+#pragma unroll 1
+    for (int kk = 0; kk < 3; ++kk) {
+      wsync();
+      const int k = 4 * P + kk;
+      const float tau = taus[k];
+      const float *vp = vptr<P>(c, kk);
+      apply<q0, s, s + 1, true>(c, a, vp, tau, kk);
+      const Reflector<float> h = reflector<P, s>(c, a, kk + 1);
+      apply<q0, s + 1, NS, false>(c, a, vp, tau, kk);
+      publish<P, s>(c, a, h, kk + 1, vptr<P>(c, kk + 1), taus + k + 1);
+    }
+    // slot s is final: write it back and start loading slot s of the next
+    // block into the same registers (its latency hides behind the rest of
+    // this block)
+    store_slot<B, s>(c, a);
+    load_slot<B + 1, s>(c, a);
+    if constexpr (s + 1 < NS) {
+      wsync();
+      const int k = 4 * P + 3;
+      const float tau = taus[k];
+      const float *vp = vptr<P>(c, 3);
+      apply<q0, s + 1, s + 2, false>(c, a, vp, tau, 3);
+      const Reflector<float> h = reflector<P + 1, s + 1>(c, a, 0);
+      apply<q0, s + 2, NS, false>(c, a, vp, tau, 3);
+      publish<P + 1, s + 1>(c, a, h, 0, vptr<P + 1>(c, 0), taus + k + 1);
+    }
+    panels<B, P + 1>(c, a);
+  }
+}
+
+template <int B>
+__device__ __forceinline__ void do_block(const Ctx &c, Tile &a) {
+  constexpr int P0 = blk_c0(B) / 4;
+  // slots beyond the previous block's width (all of block 0) load here; the
+  // others were loaded while the previous block finished
+  if constexpr (B == 0) load_slot<B, 0>(c, a);
+  if constexpr (B == 0 || blk_ns(B - 1) <= 1) load_slot<B, 1>(c, a);
+  if constexpr (B == 0 || blk_ns(B - 1) <= 2) load_slot<B, 2>(c, a);
+  if constexpr (B == 0 || blk_ns(B - 1) <= 3) load_slot<B, 3>(c, a);
+  left<B, 0>(c, a);
+  {
+    // head reflector of the block (column c0, slot 0)
+    const Reflector<float> h = reflector<P0, 0>(c, a, 0);
+    publish<P0, 0>(c, a, h, 0, vptr<P0>(c, 0), c.sm + kTauOff + 4 * P0);
+  }
+  panels<B, P0>(c, a);
+  wsync();
+}
+
+__global__ void __launch_bounds__(kThreads, 1) geqrf_ll56_kernel(LlArgs args) {
+  extern __shared__ float smem_ll[];
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int half = lane >> 4;
+  Ctx c;
+  c.lane = lane;
+  c.rg = lane & 3;
+  c.cg = (lane >> 2) & 3;
+  c.sm = smem_ll + (warp * 2 + half) * kMatWords;
+  const long long npairs = (args.batch + 1) / 2;
+  for (long long q = (long long)blockIdx.x * kWarps + warp; q < npairs; q += (long long)gridDim.x * kWarps) {
+    const long long idx = 2 * q + half;
+    // odd batch: the spare half-warp factors its neighbour's matrix again
+    // with the same instructions on the same data, so its stores write the
+    // same bits to the same addresses (no divergent branch around them)
+    const long long mi = idx < args.batch ? idx : idx - 1;
+    wsync();
+    c.Ab = args.A + mi * args.strideA + (long long)c.cg * args.lda + c.rg;
+    c.lda = args.lda;
+    Tile a;
+    do_block<0>(c, a);
+    do_block<1>(c, a);
+    do_block<2>(c, a);
+    do_block<3>(c, a);
+    {
+      const float *taus = c.sm + kTauOff;
+      float *tg = args.tau + mi * args.strideT;
+#pragma unroll
+      for (int t = lane & 15; t < kM; t += 16) tg[t] = taus[t];
+    }
+    wsync();
+  }
+}
+
+}  // namespace ll
+}  // namespace bqr

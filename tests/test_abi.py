@@ -105,7 +105,7 @@ def test_status_strings(lib):
 
 @pytest.mark.parametrize("dt,m,n,expect", [
     (0, 4, 4, "tiny"), (0, 8, 8, "tiny"), (1, 8, 8, "tiny"),
-    (0, 56, 56, "rf_f32_R4G4_14x14_x2_exact"), (1, 240, 66, "rf_c64_R32G11_8x6_cta"),
+    (0, 56, 56, "ll_f32_56x56_left4_x2"), (1, 240, 66, "rf_c64_R32G11_8x6_cta"),
     (0, 16, 16, "rf_f32"), (1, 100, 100, "rf_c64"), (0, 160, 160, "rf_f32_R16G16_10x10"),
     (0, 256, 256, "rf_f32_R32G32_8x8"), (0, 200, 64, "rf_f32_R32G8"), (1, 160, 160, "rf_c64_R16G32_10x5"), (1, 64, 64, "rf_c64_R8G8"), (0, 80, 80, "rf_f32_R8G8"),
 ])
