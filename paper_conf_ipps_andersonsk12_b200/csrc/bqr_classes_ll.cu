@@ -9,6 +9,11 @@ namespace host {
 
 int launch_ll56(const Call &c) {
   if (c.m != ll::kM || c.n != ll::kM || c.k != ll::kM || c.nrhs > 0 || c.lda < ll::kM) return BQR_ERR_NOT_SUPPORTED;
+  // the kernel moves row pairs as 8-byte words: odd lda / stride or a
+  // 4-byte-aligned base take the right-looking class of the same shape
+  const long long sA = c.strideA >= 0 ? c.strideA : (long long)c.lda * c.n;
+  if ((c.lda & 1) || (sA & 1) || (reinterpret_cast<uintptr_t>(c.A) & 7))
+    return launch_rf<float, 4, 4, 14, 14, 2, true, true, false, false>(c);
   auto kern = ll::geqrf_ll56_kernel;
   if (!ensure_smem(reinterpret_cast<const void *>(kern), ll::kSmemBytes)) return BQR_ERR_CUDA;
   if (c.resident) {
@@ -47,3 +52,9 @@ const ClassEntry *classes_ll(int *n) {
 
 }  // namespace host
 }  // namespace bqr
+
+#ifdef BQR_LL_TIMING
+extern "C" int bqr_ll_debug_stamps(void *host, size_t bytes) {
+  return cudaMemcpyFromSymbol(host, bqr::ll::g_ll_dbg, bytes) == cudaSuccess ? 0 : 2;
+}
+#endif

@@ -47,13 +47,21 @@ struct LlArgs {
 };
 
 constexpr int kM = 56;      // rows = columns
-constexpr int MP = 7;       // register-row pairs per lane: rows rg + 8p, rg + 8p + 4
+constexpr int MP = 7;       // register-row pairs per lane: rows 8p + 2rg, 8p + 2rg + 1 (8-byte loads)
 constexpr int NSMAX = 4;    // column slots per lane of a block (columns c0 + cg + 4j)
 constexpr int kWarps = 17;  // one CTA of 17 warps (34 matrices) per SM
 constexpr int kThreads = 32 * kWarps;
-// column blocks [0,16) [16,28) [28,40) [40,56)
-__host__ __device__ constexpr int blk_c0(int b) { return b == 0 ? 0 : (b == 1 ? 16 : (b == 2 ? 28 : 40)); }
-__host__ __device__ constexpr int blk_ns(int b) { return b == 0 ? 4 : (b == 1 ? 3 : (b == 2 ? 3 : 4)); }
+// column blocks (BQR_LL_PART 0: [0,16) [16,28) [28,40) [40,56);
+// 1: [0,8) [8,24) [24,40) [40,56); 2: [0,12) [12,24) [24,40) [40,56))
+#ifndef BQR_LL_PART
+#define BQR_LL_PART 2
+#endif
+constexpr int kPart = BQR_LL_PART;
+__host__ __device__ constexpr int blk_ns(int b) {
+  return kPart == 0 ? (b == 0 ? 4 : (b == 1 ? 3 : (b == 2 ? 3 : 4)))
+                    : (kPart == 1 ? (b == 0 ? 2 : 4) : (b <= 1 ? 3 : 4));
+}
+__host__ __device__ constexpr int blk_c0(int b) { return b == 0 ? 0 : blk_c0(b - 1) + 4 * blk_ns(b - 1); }
 constexpr int kNB = 4;
 // reflectors of panels 0..9 (columns 0..39) are kept for the left-looking
 // applies; panel P's vector holds this lane's pairs P/2 .. MP-1
@@ -85,11 +93,30 @@ __device__ __forceinline__ void sts64(float *p, float2 v) {
   asm volatile("st.shared.v2.f32 [%0], {%1,%2};" ::"r"(s), "f"(v.x), "f"(v.y) : "memory");
 }
 
+#ifdef BQR_LL_TIMING
+// debug builds only: clock64 stamps of CTA 0's warps (first matrix pair):
+// [warp][event], events 3B = block B start, 3B+1 after its left-looking
+// applies, 3B+2 after its panels, 12 = end of the matrix
+constexpr int kDbgEv = 13;
+static __device__ unsigned long long g_ll_dbg[kWarps * kDbgEv];
+#define LL_STAMP(c, e)                                                              \
+  do {                                                                              \
+    if (blockIdx.x == 0 && (c).lane == 0 && (c).first) g_ll_dbg[(threadIdx.x >> 5) * kDbgEv + (e)] = clock64(); \
+  } while (0)
+#else
+#define LL_STAMP(c, e) \
+  do {                 \
+  } while (0)
+#endif
+
 struct Ctx {
   float *sm;    // this matrix's shared words
   float *Ab;    // this lane's element (rg, cg) of the matrix in global memory
   int lda;
   int rg, cg, lane;
+#ifdef BQR_LL_TIMING
+  bool first;
+#endif
 };
 
 // this lane's vector of reflector k = 4P + kk, positioned at pair P/2
@@ -104,23 +131,25 @@ __device__ __forceinline__ float *vptr(const Ctx &c, int kk) {
 
 using Tile = float2[MP][NSMAX];
 
+#ifndef BQR_LL_UNROLL_LEFT
+#define BQR_LL_UNROLL_LEFT 4
+#endif
+constexpr int kUnrollLeft = BQR_LL_UNROLL_LEFT;
+
 // slot j of block B (columns c0 + cg + 4j, rows rg + 4i) <-> HBM
 template <int B, int J>
 __device__ __forceinline__ void load_slot(const Ctx &c, Tile &a) {
   if constexpr (B < kNB && J < blk_ns(B)) {
     const float *col = c.Ab + (long long)(blk_c0(B) + 4 * J) * c.lda;
 #pragma unroll
-    for (int p = 0; p < MP; ++p) a[p][J] = make_float2(col[8 * p], col[8 * p + 4]);
+    for (int p = 0; p < MP; ++p) a[p][J] = *reinterpret_cast<const float2 *>(col + 8 * p);
   }
 }
 template <int B, int J>
 __device__ __forceinline__ void store_slot(const Ctx &c, const Tile &a) {
   float *col = c.Ab + (long long)(blk_c0(B) + 4 * J) * c.lda;
 #pragma unroll
-  for (int p = 0; p < MP; ++p) {
-    col[8 * p] = a[p][J].x;
-    col[8 * p + 4] = a[p][J].y;
-  }
+  for (int p = 0; p < MP; ++p) *reinterpret_cast<float2 *>(col + 8 * p) = a[p][J];
 }
 
 
@@ -176,14 +205,12 @@ __device__ __forceinline__ Reflector<float> reflector(const Ctx &c, const Tile &
   for (int p = q0; p < MP; ++p) {
     float2 x = a[p][S];
     if (p == q0) {
-      if constexpr (PP % 2 == 0) {
-        alpha = c.rg == kkn ? x.x : 0.f;
-        x.x = c.rg > kkn ? x.x : 0.f;
-      } else {
-        alpha = c.rg == kkn ? x.y : 0.f;
-        x.y = c.rg > kkn ? x.y : 0.f;
-        x.x = 0.f;
-      }
+      // pair q0 holds rows 8 q0 + 2 rg (x) and + 1 (y); the pivot is row
+      // 8 q0 + kr
+      const int kr = 4 * (PP % 2) + kkn;
+      alpha = 2 * c.rg == kr ? x.x : (2 * c.rg + 1 == kr ? x.y : 0.f);
+      x.x = 2 * c.rg > kr ? x.x : 0.f;
+      x.y = 2 * c.rg + 1 > kr ? x.y : 0.f;
     }
     acc[(p - q0) & 1] = __ffma2_rn(x, x, acc[(p - q0) & 1]);
   }
@@ -191,7 +218,7 @@ __device__ __forceinline__ Reflector<float> reflector(const Ctx &c, const Tile &
   float sig = accs.x + accs.y;
   sig += __shfl_xor_sync(0xffffffffu, sig, 1);
   sig += __shfl_xor_sync(0xffffffffu, sig, 2);
-  alpha = __shfl_sync(0xffffffffu, alpha, (c.lane & ~3) | kkn);
+  alpha = __shfl_sync(0xffffffffu, alpha, (c.lane & ~3) | ((4 * (PP % 2) + kkn) >> 1));
   return make_reflector(alpha, sig);
 }
 
@@ -207,18 +234,14 @@ __device__ __forceinline__ void publish(const Ctx &c, Tile &a, const Reflector<f
 #pragma unroll
   for (int p = q0; p < MP; ++p) {
     const float2 x = a[p][S];
-    const float2 xs = make_float2(x.x * scal, x.y * scal);
+    const float2 xs = __fmul2_rn(x, make_float2(scal, scal));
     float2 v = xs, nx = xs;
     if (p == q0) {
-      if constexpr (PP % 2 == 0) {
-        v.x = c.rg > kkn ? xs.x : (c.rg == kkn ? 1.f : 0.f);
-        nx.x = c.rg > kkn ? xs.x : ((own && c.rg == kkn) ? h.beta : x.x);
-      } else {
-        v.x = 0.f;
-        nx.x = x.x;
-        v.y = c.rg > kkn ? xs.y : (c.rg == kkn ? 1.f : 0.f);
-        nx.y = c.rg > kkn ? xs.y : ((own && c.rg == kkn) ? h.beta : x.y);
-      }
+      const int kr = 4 * (PP % 2) + kkn, r0 = 2 * c.rg, r1 = 2 * c.rg + 1;
+      v.x = r0 > kr ? xs.x : (r0 == kr ? 1.f : 0.f);
+      nx.x = r0 > kr ? xs.x : ((own && r0 == kr) ? h.beta : x.x);
+      v.y = r1 > kr ? xs.y : (r1 == kr ? 1.f : 0.f);
+      nx.y = r1 > kr ? xs.y : ((own && r1 == kr) ? h.beta : x.y);
     }
     a[p][S] = nx;
     if (own) *reinterpret_cast<float2 *>(vdst + 2 * (p - q0)) = v;
@@ -232,7 +255,7 @@ template <int B, int P>
 __device__ __forceinline__ void left(const Ctx &c, Tile &a) {
   if constexpr (P < blk_c0(B) / 4) {
     const float *taus = c.sm + kTauOff;
-#pragma unroll 1
+#pragma unroll kUnrollLeft
     for (int kk = 0; kk < 4; ++kk) apply<P / 2, 0, blk_ns(B), false>(c, a, vptr<P>(c, kk), taus[4 * P + kk], kk);
     left<B, P + 1>(c, a);
   }
@@ -281,11 +304,13 @@ __device__ __forceinline__ void do_block(const Ctx &c, Tile &a) {
   constexpr int P0 = blk_c0(B) / 4;
   // slots beyond the previous block's width (all of block 0) load here; the
   // others were loaded while the previous block finished
+  LL_STAMP(c, 3 * B);
   if constexpr (B == 0) load_slot<B, 0>(c, a);
   if constexpr (B == 0 || blk_ns(B - 1) <= 1) load_slot<B, 1>(c, a);
   if constexpr (B == 0 || blk_ns(B - 1) <= 2) load_slot<B, 2>(c, a);
   if constexpr (B == 0 || blk_ns(B - 1) <= 3) load_slot<B, 3>(c, a);
   left<B, 0>(c, a);
+  LL_STAMP(c, 3 * B + 1);
   {
     // head reflector of the block (column c0, slot 0)
     const Reflector<float> h = reflector<P0, 0>(c, a, 0);
@@ -293,17 +318,25 @@ __device__ __forceinline__ void do_block(const Ctx &c, Tile &a) {
   }
   panels<B, P0>(c, a);
   wsync();
+  LL_STAMP(c, 3 * B + 2);
 }
 
 __global__ void __launch_bounds__(kThreads, 1) geqrf_ll56_kernel(LlArgs args) {
   extern __shared__ float smem_ll[];
-  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  // the warp index through a shuffle: provably warp-uniform, so the matrix
+  // loop below is a uniform branch (otherwise ptxas guards every later
+  // shuffle with a divergence check, BRA.DIV, that splits the basic blocks
+  // the scheduler interleaves the reflector chain across)
+  const int lane = threadIdx.x & 31, warp = __shfl_sync(0xffffffffu, (int)(threadIdx.x >> 5), 0);
   const int half = lane >> 4;
   Ctx c;
   c.lane = lane;
   c.rg = lane & 3;
   c.cg = (lane >> 2) & 3;
   c.sm = smem_ll + (warp * 2 + half) * kMatWords;
+#ifdef BQR_LL_TIMING
+  c.first = true;
+#endif
   const long long npairs = (args.batch + 1) / 2;
   for (long long q = (long long)blockIdx.x * kWarps + warp; q < npairs; q += (long long)gridDim.x * kWarps) {
     const long long idx = 2 * q + half;
@@ -312,7 +345,7 @@ __global__ void __launch_bounds__(kThreads, 1) geqrf_ll56_kernel(LlArgs args) {
     // same bits to the same addresses (no divergent branch around them)
     const long long mi = idx < args.batch ? idx : idx - 1;
     wsync();
-    c.Ab = args.A + mi * args.strideA + (long long)c.cg * args.lda + c.rg;
+    c.Ab = args.A + mi * args.strideA + (long long)c.cg * args.lda + 2 * c.rg;
     c.lda = args.lda;
     Tile a;
     do_block<0>(c, a);
@@ -326,6 +359,10 @@ __global__ void __launch_bounds__(kThreads, 1) geqrf_ll56_kernel(LlArgs args) {
       for (int t = lane & 15; t < kM; t += 16) tg[t] = taus[t];
     }
     wsync();
+    LL_STAMP(c, 12);
+#ifdef BQR_LL_TIMING
+    c.first = false;
+#endif
   }
 }
 
