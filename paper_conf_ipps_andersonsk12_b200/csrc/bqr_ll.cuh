@@ -135,6 +135,9 @@ using Tile = float2[MP][NSMAX];
 #define BQR_LL_UNROLL_LEFT 4
 #endif
 constexpr int kUnrollLeft = BQR_LL_UNROLL_LEFT;
+#ifndef BQR_LL_PACKRED
+#define BQR_LL_PACKRED 1
+#endif
 
 // slot j of block B (columns c0 + cg + 4j, rows rg + 4i) <-> HBM
 template <int B, int J>
@@ -169,6 +172,40 @@ __device__ __forceinline__ void apply(const Ctx &c, Tile &a, const float *vp, fl
     for (int p = Q0; p < MP; ++p)
 #pragma unroll
       for (int j = 0; j < NS; ++j) w[j] = __ffma2_rn(v[p], a[p][J0 + j], w[j]);
+    float2 nt[NS];
+#if BQR_LL_PACKRED
+    // column pairs packed for the FP32 pipe: (w_j.x + w_j.y, w_j+1.x + w_j+1.y)
+    // as one FADD2, the butterfly adds as FADD2, -tau * s as FMUL2
+    constexpr int NP = (NS + 1) / 2;
+    float2 sp[NP];
+#pragma unroll
+    for (int q = 0; q < NP; ++q) {
+      if (2 * q + 1 < NS)
+        sp[q] = __fadd2_rn(make_float2(w[2 * q].x, w[2 * q + 1].x), make_float2(w[2 * q].y, w[2 * q + 1].y));
+      else
+        sp[q] = make_float2(w[2 * q].x + w[2 * q].y, 0.f);
+    }
+#pragma unroll
+    for (int o = 1; o <= 2; o <<= 1) {
+#pragma unroll
+      for (int q = 0; q < NP; ++q) {
+        if (2 * q + 1 < NS) {
+          const float2 r = make_float2(__shfl_xor_sync(0xffffffffu, sp[q].x, o), __shfl_xor_sync(0xffffffffu, sp[q].y, o));
+          sp[q] = __fadd2_rn(sp[q], r);
+        } else {
+          sp[q].x += __shfl_xor_sync(0xffffffffu, sp[q].x, o);
+        }
+      }
+    }
+#pragma unroll
+    for (int q = 0; q < NP; ++q) {
+      const float2 t = __fmul2_rn(sp[q], make_float2(-tau, -tau));
+      float t0 = t.x;
+      if (MASK0 && q == 0) t0 = c.cg > kk ? t0 : 0.f;
+      nt[2 * q] = make_float2(t0, t0);
+      if (2 * q + 1 < NS) nt[2 * q + 1] = make_float2(t.y, t.y);
+    }
+#else
     float s[NS];
 #pragma unroll
     for (int j = 0; j < NS; ++j) s[j] = w[j].x + w[j].y;
@@ -176,13 +213,13 @@ __device__ __forceinline__ void apply(const Ctx &c, Tile &a, const float *vp, fl
     for (int j = 0; j < NS; ++j) s[j] += __shfl_xor_sync(0xffffffffu, s[j], 1);
 #pragma unroll
     for (int j = 0; j < NS; ++j) s[j] += __shfl_xor_sync(0xffffffffu, s[j], 2);
-    float2 nt[NS];
 #pragma unroll
     for (int j = 0; j < NS; ++j) {
       float t = tau * s[j];
       if (MASK0 && j == 0) t = c.cg > kk ? t : 0.f;
       nt[j] = make_float2(-t, -t);
     }
+#endif
 #ifdef BQR_LL_RELOAD
 #pragma unroll
     for (int p = Q0; p < MP; ++p) v[p] = lds64(vp + 2 * (p - Q0));
