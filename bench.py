@@ -112,12 +112,19 @@ class ClockSampler:
         return {"sm_mhz": med, "sm_max_mhz": self.max_mhz, "reasons": names, "samples": len(self.samples)}
 
 
-def load_traffic(name: str):
+def load_traffic(name: str, kernel: str | None = None):
+    """DRAM bytes per launch of config `name` from the committed ncu capture;
+    None when the capture was taken of another kernel class than the one the
+    dispatch picks now."""
     try:
         with open(PROFILE_TRAFFIC) as f:
-            return json.load(f).get(name)
+            t = json.load(f)
     except OSError:
         return None
+    cls = t.get("_detail", {}).get(name, {}).get("class")
+    if kernel is not None and cls is not None and cls != kernel:
+        return None
+    return t.get(name)
 
 
 # --------------------------------------------------------------------- GPU arm
@@ -298,7 +305,11 @@ def roofline_obj(w: Workload, qr_ms: float, peaks: dict, n_sm: int, fused: bool 
     nbytes = w.bytes + (w.bytes_apply if fused else 0)
     t_roof, bound = bm.roofline_time_s(flops, nbytes, hbm, fp32)
     t = qr_ms / 1e3
-    traffic = load_traffic(w.name)
+    kname = ({"lu": "lu_rf_kernel (LU, no pivoting)", "gj": "lu_rf_kernel (Gauss-Jordan)"}[w.kind]
+             if w.kind != "qr" else
+             w.bqr.load().bqr_qhb_kernel_name(w.code, w.m, w.n, w.nrhs).decode() if fused
+             else w.bqr.kernel_name(w.code, w.m, w.n))
+    traffic = load_traffic(w.name, kname)
     if bound == "hbm":
         ach, peak, unit = nbytes / t / 1e9, hbm, "GB/s"
     else:
@@ -309,10 +320,7 @@ def roofline_obj(w: Workload, qr_ms: float, peaks: dict, n_sm: int, fused: bool 
                             f"derived: {n_sm} SMs x 128 FP32 lanes x 2 x {peaks.get('sm_max_mhz', 1965.0)} MHz"),
             "roofline_us": round(t_roof * 1e6, 3), "kernel_us": round(qr_ms * 1e3, 3),
             "algorithmic_bytes": nbytes, "useful_flops": flops,
-            "kernel": ({"lu": "lu_rf_kernel (LU, no pivoting)", "gj": "lu_rf_kernel (Gauss-Jordan)"}[w.kind]
-                       if w.kind != "qr" else
-                       w.bqr.load().bqr_qhb_kernel_name(w.code, w.m, w.n, w.nrhs).decode() if fused
-                       else w.bqr.kernel_name(w.code, w.m, w.n))}
+            "kernel": kname}
 
 
 def e2e_host(w: Workload, steps: int, warmup: int, torch, dist, world):

@@ -135,6 +135,9 @@ using Tile = float2[MP][NSMAX];
 #define BQR_LL_UNROLL_LEFT 4
 #endif
 constexpr int kUnrollLeft = BQR_LL_UNROLL_LEFT;
+#ifndef BQR_LL_LOADLAG
+#define BQR_LL_LOADLAG 0
+#endif
 #ifndef BQR_LL_PACKRED
 #define BQR_LL_PACKRED 1
 #endif
@@ -321,7 +324,14 @@ __device__ __forceinline__ void panels(const Ctx &c, Tile &a) {
     // block into the same registers (its latency hides behind the rest of
     // this block)
     store_slot<B, s>(c, a);
+#if BQR_LL_LOADLAG
+    // one panel later: the store has read the registers by then (no WAR
+    // stall of the load behind the store queue)
+    if constexpr (s >= 1) load_slot<B + 1, s - 1>(c, a);
+    if constexpr (s + 1 == NS) load_slot<B + 1, s>(c, a);
+#else
     load_slot<B + 1, s>(c, a);
+#endif
     if constexpr (s + 1 < NS) {
       wsync();
       const int k = 4 * P + 3;

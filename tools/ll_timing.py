@@ -19,7 +19,7 @@ import paper_conf_ipps_andersonsk12_b200 as bqr  # noqa: E402
 bqr._LIB_PATH = os.path.abspath(sys.argv[1])
 lib = bqr.load()
 W, E = 17, 13
-w = bench.Workload("C3", 0, 1, torch, bqr)
+w = bench.Workload("C3", 0, 1, torch, bqr, batch=int(sys.argv[2]) if len(sys.argv) > 2 else None)
 for _ in range(3):
     w.restore()
     torch.cuda.synchronize()
@@ -28,6 +28,8 @@ for _ in range(3):
 buf = np.zeros(W * E, dtype=np.uint64)
 assert lib.bqr_ll_debug_stamps(buf.ctypes.data_as(ctypes.c_void_p), ctypes.c_size_t(buf.nbytes)) == 0
 st = buf.reshape(W, E).astype(np.int64)
+st = st[st[:, 0] > 0]
+W = st.shape[0]
 t0 = st[:, 0].min()
 rel = st - t0
 print("warp " + " ".join(f"{n:>7s}" for n in ["b0", "b0L", "b0P", "b1", "b1L", "b1P", "b2", "b2L", "b2P", "b3", "b3L", "b3P", "end"]))
