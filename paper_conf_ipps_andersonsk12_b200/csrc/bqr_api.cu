@@ -61,16 +61,17 @@ using namespace bqr::host;
 // classes, then fp32, then complex64, then the
 // experiment-only alternatives (BQR_FORCE_VARIANT).
 struct Tables {
-  static constexpr int kN = 6;
+  static constexpr int kN = 7;
   const ClassEntry *t[kN];
   int n[kN];
   Tables() {
     t[0] = classes_ll(&n[0]);
-    t[1] = classes_co(&n[1]);
-    t[2] = classes_headline(&n[2]);
-    t[3] = classes_f32(&n[3]);
-    t[4] = classes_c64(&n[4]);
-    t[5] = classes_alt(&n[5]);
+    t[1] = classes_llc(&n[1]);
+    t[2] = classes_co(&n[2]);
+    t[3] = classes_headline(&n[3]);
+    t[4] = classes_f32(&n[4]);
+    t[5] = classes_c64(&n[5]);
+    t[6] = classes_alt(&n[6]);
   }
   template <class F>
   const Plan *find(F pred) const {
@@ -129,6 +130,9 @@ const Plan *pick_fused(bqr_dtype_t dt, int m, int n, int nrhs) {
     if (e.dt != dt || m > e.mmax || n + nrhs > e.nmax) return;
     if (std::strncmp(e.plan.name, "alt_", 4) == 0) return;  // experiment-only variants (BQR_FORCE_VARIANT)
     if (!std::strstr(e.plan.name, "_aug")) return;
+    // exact-shape fused classes (bounds == exact shape) only for that shape
+    if (e.exact_m > 0 && e.mmax == e.exact_m && e.nmax == e.exact_n && (e.exact_m != m || e.exact_n != n + nrhs))
+      return;
     const int area = e.mmax * e.nmax;
     if (area < best_area) {
       best = &e.plan;

@@ -81,6 +81,21 @@ static_assert(kMatWords % 2 == 0, "8-byte aligned vectors");
 static_assert(kSmemBytes <= 232448, "one CTA of 34 matrices per SM");
 static_assert(blk_c0(kNB - 1) == 4 * kKeepP && blk_c0(kNB - 1) + 4 * blk_ns(kNB - 1) == kM, "blocks");
 
+// packed FP32 (one fma.rn.f32x2 per row pair) or two scalar FMAs: on B200
+// one warp issues an FFMA2 every ~2.8 cycles but a 3-register FFMA every
+// ~1.1 (tools/micro/ffma2_rate.cu: 23 vs 29 FMA/clk per scheduler), so for
+// a latency-bound warp the scalar form is faster
+#ifndef BQR_LL_FFMA2
+#define BQR_LL_FFMA2 1
+#endif
+__device__ __forceinline__ float2 fma2(float2 a, float2 b, float2 c) {
+#if BQR_LL_FFMA2
+  return __ffma2_rn(a, b, c);
+#else
+  return make_float2(fmaf(a.x, b.x, c.x), fmaf(a.y, b.y, c.y));
+#endif
+}
+
 __device__ __forceinline__ void wsync() { asm volatile("bar.warp.sync -1;" ::: "memory"); }
 __device__ __forceinline__ float2 lds64(const float *p) {
   float2 v;
@@ -174,7 +189,7 @@ __device__ __forceinline__ void apply(const Ctx &c, Tile &a, const float *vp, fl
 #pragma unroll
     for (int p = Q0; p < MP; ++p)
 #pragma unroll
-      for (int j = 0; j < NS; ++j) w[j] = __ffma2_rn(v[p], a[p][J0 + j], w[j]);
+      for (int j = 0; j < NS; ++j) w[j] = fma2(v[p], a[p][J0 + j], w[j]);
     float2 nt[NS];
 #if BQR_LL_PACKRED
     // column pairs packed for the FP32 pipe: (w_j.x + w_j.y, w_j+1.x + w_j+1.y)
@@ -230,7 +245,7 @@ __device__ __forceinline__ void apply(const Ctx &c, Tile &a, const float *vp, fl
 #pragma unroll
     for (int p = Q0; p < MP; ++p)
 #pragma unroll
-      for (int j = 0; j < NS; ++j) a[p][J0 + j] = __ffma2_rn(v[p], nt[j], a[p][J0 + j]);
+      for (int j = 0; j < NS; ++j) a[p][J0 + j] = fma2(v[p], nt[j], a[p][J0 + j]);
   }
 }
 
@@ -252,7 +267,7 @@ __device__ __forceinline__ Reflector<float> reflector(const Ctx &c, const Tile &
       x.x = 2 * c.rg > kr ? x.x : 0.f;
       x.y = 2 * c.rg + 1 > kr ? x.y : 0.f;
     }
-    acc[(p - q0) & 1] = __ffma2_rn(x, x, acc[(p - q0) & 1]);
+    acc[(p - q0) & 1] = fma2(x, x, acc[(p - q0) & 1]);
   }
   const float2 accs = __fadd2_rn(acc[0], acc[1]);
   float sig = accs.x + accs.y;
