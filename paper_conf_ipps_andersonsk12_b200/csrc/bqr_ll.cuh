@@ -74,7 +74,10 @@ constexpr int kRingOff = kVStore;           // 2 x [4 row lanes][pairs kRingQ..6
 constexpr int kRingLen = 2 * (MP - kRingQ);
 constexpr int kRingBuf = 4 * kRingLen;
 constexpr int kTauOff = kRingOff + 2 * kRingBuf;
-constexpr int kMatWords = kTauOff + kM;     // 1688 words: 34 matrices = 224 KB
+// g_k = v_{k+1}^T v_k for the reflector pairs (k, k+1), k even < 4 kKeepP,
+// of the paired left-looking applies
+constexpr int kGOff = kTauOff + kM;
+constexpr int kMatWords = kGOff + 2 * kKeepP;  // 1708 words: 34 matrices = 227 KB
 constexpr size_t kSmemBytes = (size_t)kWarps * 2 * kMatWords * 4;
 static_assert(NSMAX == 4, "do_block loads slots 0..3");
 static_assert(kMatWords % 2 == 0, "8-byte aligned vectors");
@@ -150,6 +153,12 @@ using Tile = float2[MP][NSMAX];
 #define BQR_LL_UNROLL_LEFT 4
 #endif
 constexpr int kUnrollLeft = BQR_LL_UNROLL_LEFT;
+// paired left-looking applies (one reduction for H_k, H_{k+1}): parity
+// green but slower on B200 (81.4 vs 69.6 us: 484 B of spills at the
+// 96-register cap), off
+#ifndef BQR_LL_PAIR
+#define BQR_LL_PAIR 0
+#endif
 #ifndef BQR_LL_LOADLAG
 #define BQR_LL_LOADLAG 0
 #endif
@@ -306,13 +315,90 @@ __device__ __forceinline__ void publish(const Ctx &c, Tile &a, const Reflector<f
 
 // ---------------------------------------------------------------- phases
 // left-looking: H_0 .. H_{c0-1} (panels 0 .. c0/4 - 1) on block B
+// H_{k+1} H_k on slots [0, NS) in one pass (k even, both of panel P, rows
+// from pair Q0): with w = v_k^T A, w' = v_{k+1}^T A (ONE reduction for both)
+// and g = v_{k+1}^T v_k, H_{k+1} H_k A = A - v_k t^T - v_{k+1} t'^T where
+// t = tau_k w and t' = tau_{k+1} (w' - g t)
+template <int Q0, int NS>
+__device__ __forceinline__ void apply_pair(const Ctx &c, Tile &a, const float *vp0, const float *vp1, float tau0,
+                                           float tau1, float g) {
+  float2 w0[NS], w1[NS];
+#pragma unroll
+  for (int j = 0; j < NS; ++j) w0[j] = w1[j] = make_float2(0.f, 0.f);
+#pragma unroll
+  for (int p = Q0; p < MP; ++p) {
+    const float2 v0 = lds64(vp0 + 2 * (p - Q0)), v1 = lds64(vp1 + 2 * (p - Q0));
+#pragma unroll
+    for (int j = 0; j < NS; ++j) {
+      w0[j] = fma2(v0, a[p][j], w0[j]);
+      w1[j] = fma2(v1, a[p][j], w1[j]);
+    }
+  }
+  float2 sp[NS];  // (v_k^T a_j, v_{k+1}^T a_j)
+#pragma unroll
+  for (int j = 0; j < NS; ++j)
+    sp[j] = __fadd2_rn(make_float2(w0[j].x, w1[j].x), make_float2(w0[j].y, w1[j].y));
+#pragma unroll
+  for (int o = 1; o <= 2; o <<= 1)
+#pragma unroll
+    for (int j = 0; j < NS; ++j)
+      sp[j] = __fadd2_rn(sp[j], make_float2(__shfl_xor_sync(0xffffffffu, sp[j].x, o),
+                                            __shfl_xor_sync(0xffffffffu, sp[j].y, o)));
+  float2 n0[NS], n1[NS];
+#pragma unroll
+  for (int j = 0; j < NS; ++j) {
+    const float t0 = tau0 * sp[j].x;
+    const float t1 = tau1 * fmaf(-g, t0, sp[j].y);
+    n0[j] = make_float2(-t0, -t0);
+    n1[j] = make_float2(-t1, -t1);
+  }
+#pragma unroll
+  for (int p = Q0; p < MP; ++p) {
+    const float2 v0 = lds64(vp0 + 2 * (p - Q0)), v1 = lds64(vp1 + 2 * (p - Q0));
+#pragma unroll
+    for (int j = 0; j < NS; ++j) a[p][j] = fma2(v1, n1[j], fma2(v0, n0[j], a[p][j]));
+  }
+}
+
 template <int B, int P>
 __device__ __forceinline__ void left(const Ctx &c, Tile &a) {
   if constexpr (P < blk_c0(B) / 4) {
     const float *taus = c.sm + kTauOff;
+#if BQR_LL_PAIR
+#pragma unroll
+    for (int kk = 0; kk < 4; kk += 2)
+      apply_pair<P / 2, blk_ns(B)>(c, a, vptr<P>(c, kk), vptr<P>(c, kk + 1), taus[4 * P + kk], taus[4 * P + kk + 1],
+                                   c.sm[kGOff + 2 * P + kk / 2]);
+#else
 #pragma unroll kUnrollLeft
     for (int kk = 0; kk < 4; ++kk) apply<P / 2, 0, blk_ns(B), false>(c, a, vptr<P>(c, kk), taus[4 * P + kk], kk);
+#endif
     left<B, P + 1>(c, a);
+  }
+}
+
+// g_k = v_{k+1}^T v_k of the pairs (k, k+1) of panel P (k = 4P, 4P + 2),
+// written by lane (rg 0, cg 0) of the matrix
+template <int P>
+__device__ __forceinline__ void gram_pairs(const Ctx &c) {
+  constexpr int Q0 = P / 2;
+#pragma unroll
+  for (int kk = 0; kk < 4; kk += 2) {
+    const float *vp0 = vptr<P>(c, kk), *vp1 = vptr<P>(c, kk + 1);
+    float2 acc = make_float2(0.f, 0.f);
+#pragma unroll
+    for (int p = Q0; p < MP; ++p) acc = fma2(lds64(vp0 + 2 * (p - Q0)), lds64(vp1 + 2 * (p - Q0)), acc);
+    float g = acc.x + acc.y;
+    g += __shfl_xor_sync(0xffffffffu, g, 1);
+    g += __shfl_xor_sync(0xffffffffu, g, 2);
+    if (c.rg == 0 && c.cg == 0) c.sm[kGOff + 2 * P + kk / 2] = g;
+  }
+}
+template <int P, int PE>
+__device__ __forceinline__ void gram_block(const Ctx &c) {
+  if constexpr (P < PE && P < kKeepP) {
+    gram_pairs<P>(c);
+    gram_block<P + 1, PE>(c);
   }
 }
 
@@ -380,6 +466,11 @@ __device__ __forceinline__ void do_block(const Ctx &c, Tile &a) {
   }
   panels<B, P0>(c, a);
   wsync();
+#if BQR_LL_PAIR
+  // the pair products g of this block's reflectors, for the later blocks
+  gram_block<P0, P0 + blk_ns(B)>(c);
+  wsync();
+#endif
   LL_STAMP(c, 3 * B + 2);
 }
 
