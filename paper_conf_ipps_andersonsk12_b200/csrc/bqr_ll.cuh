@@ -46,6 +46,12 @@ struct LlArgs {
   long long strideA, strideT;
 };
 
+// paired left-looking applies (one reduction for H_k, H_{k+1}): parity
+// green but slower on B200 (81.4 vs 69.6 us: 484 B of spills at the
+// 96-register cap), off
+#ifndef BQR_LL_PAIR
+#define BQR_LL_PAIR 0
+#endif
 constexpr int kM = 56;      // rows = columns
 constexpr int MP = 7;       // register-row pairs per lane: rows 8p + 2rg, 8p + 2rg + 1 (8-byte loads)
 constexpr int NSMAX = 4;    // column slots per lane of a block (columns c0 + cg + 4j)
@@ -77,7 +83,7 @@ constexpr int kTauOff = kRingOff + 2 * kRingBuf;
 // g_k = v_{k+1}^T v_k for the reflector pairs (k, k+1), k even < 4 kKeepP,
 // of the paired left-looking applies
 constexpr int kGOff = kTauOff + kM;
-constexpr int kMatWords = kGOff + 2 * kKeepP;  // 1708 words: 34 matrices = 227 KB
+constexpr int kMatWords = kGOff + (BQR_LL_PAIR ? 2 * kKeepP : 0);  // 1688 (1708) words: 34 matrices = 224 (227) KB
 constexpr size_t kSmemBytes = (size_t)kWarps * 2 * kMatWords * 4;
 static_assert(NSMAX == 4, "do_block loads slots 0..3");
 static_assert(kMatWords % 2 == 0, "8-byte aligned vectors");
@@ -153,12 +159,6 @@ using Tile = float2[MP][NSMAX];
 #define BQR_LL_UNROLL_LEFT 4
 #endif
 constexpr int kUnrollLeft = BQR_LL_UNROLL_LEFT;
-// paired left-looking applies (one reduction for H_k, H_{k+1}): parity
-// green but slower on B200 (81.4 vs 69.6 us: 484 B of spills at the
-// 96-register cap), off
-#ifndef BQR_LL_PAIR
-#define BQR_LL_PAIR 0
-#endif
 #ifndef BQR_LL_LOADLAG
 #define BQR_LL_LOADLAG 0
 #endif
