@@ -31,8 +31,7 @@ int launch_ll56(const Call &c) {
   int sms = 0, bps = 0;
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, current_device());
   cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, kern, ll::kThreads, ll::kSmemBytes);
-  long long grid = (pairs + ll::kWarps - 1) / ll::kWarps;
-  grid = std::min<long long>(grid, (long long)sms * std::max(1, bps));
+  const long long grid = std::min<long long>(pairs, (long long)sms * std::max(1, bps));
   if (grid <= 0) return BQR_SUCCESS;
   kern<<<(unsigned)grid, ll::kThreads, ll::kSmemBytes, c.stream>>>(a);
   return finish_launch();

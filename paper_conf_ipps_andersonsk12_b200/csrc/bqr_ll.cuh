@@ -491,7 +491,14 @@ __global__ void __launch_bounds__(kThreads, 1) geqrf_ll56_kernel(LlArgs args) {
   c.first = true;
 #endif
   const long long npairs = (args.batch + 1) / 2;
-  for (long long q = (long long)blockIdx.x * kWarps + warp; q < npairs; q += (long long)gridDim.x * kWarps) {
+  // CTA b owns the contiguous pairs [b chunk, (b + 1) chunk), chunk =
+  // ceil(pairs / grid) with grid = min(pairs, SMs): a full batch gives 17
+  // pairs per SM as before, a batch smaller than one resident round spreads
+  // over all SMs (one warp per SM first) instead of filling few SMs
+  const long long chunk = (npairs + gridDim.x - 1) / gridDim.x;
+  for (long long wq = warp; wq < chunk; wq += kWarps) {
+    const long long q = (long long)blockIdx.x * chunk + wq;
+    if (q >= npairs) break;
     const long long idx = 2 * q + half;
     // odd batch: the spare half-warp factors its neighbour's matrix again
     // with the same instructions on the same data, so its stores write the
