@@ -160,6 +160,12 @@ C3_LAYOUT = Layout(m=56, n=56, R=4, G=4, MR=14, NC=14, cplx=False, resident=16, 
                    overhead=110.0)
 C4_LAYOUT = Layout(m=240, n=66, R=32, G=11, MR=8, NC=6, cplx=True, resident=1, warps_per_matrix=11,
                    overhead=90.0, packed=True, signal=60.0)
+# round 2: the left-looking C3 class (csrc/bqr_ll.cuh) -- the same 4 x 4
+# lanes per matrix and per-column reflector chain, but only a <= 4-slot
+# column block per lane and 34 matrices resident per SM (one round)
+C3_LL_LAYOUT = Layout(m=56, n=56, R=4, G=4, MR=14, NC=4, cplx=False, resident=34, warps_per_matrix=0.5,
+                      overhead=110.0, packed=True)
+LAYOUTS = {"C3": C3_LAYOUT, "C3_LL": C3_LL_LAYOUT, "C4": C4_LAYOUT}
 
 
 # ----------------------------------------------------------------------------

@@ -50,6 +50,7 @@ def test_r02_bounds_bracket_the_measurements():
             assert f["lo"] <= f["measured_batch_1"] <= f["hi"], (cfg, f)
     # the recomputation agrees with the file
     import bqr_model as M
-    b = M.bounds_us(M.C3_LAYOUT, 5000, d["C3"]["ncu"]["executed_instructions"], d["C3"]["ncu"]["warp_cpi"],
+    b = M.bounds_us(M.LAYOUTS[d["C3"].get("layout", "C3")], 5000, d["C3"]["ncu"]["executed_instructions"],
+                    d["C3"]["ncu"]["warp_cpi"],
                     5000 * 117077.33333333333)
     assert abs(b["lo_us"] - d["C3"]["lo_us"]) < 1e-6 and abs(b["hi_us"] - d["C3"]["hi_us"]) < 1e-6
