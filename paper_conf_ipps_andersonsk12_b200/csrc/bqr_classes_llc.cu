@@ -45,10 +45,10 @@ int launch_llc240(const Call &c) {
 
 namespace {
 const ClassEntry kTable[] = {
-    // experiment (BQR_FORCE_VARIANT): equal to the right-looking class on
-    // B200 (geqrf 121.4 vs 117.7 us, fused step 121.0 vs ~119 us) -- two
-    // matrices per SM, but each column step's owner chain (30 rows per lane)
-    // is twice as long (profiles/r02/experiments/README.md)
+    // experiment (BQR_FORCE_VARIANT): two matrices per SM, decoupled per-
+    // reflector mbarriers; parity green but equal to the right-looking class
+    // on B200 (geqrf 119.3 vs 118.1 us, fused step 119.4 vs ~119 us; an
+    // 8-row-lane CTA-barrier version: 121.4): profiles/r02/experiments/README.md
     {BQR_C64, 240, 66, 240, 66, true,
      Plan{"alt_llc_c64_240x66_left3", &launch_llc240, &launch_rf<float2, 32, 11, 8, 6, 1, false, false, false, true>}},
     // the fused [A | b] step of C4 (picked by pick_fused for exactly 240 x (66 + 1))

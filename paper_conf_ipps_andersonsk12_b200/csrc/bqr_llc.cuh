@@ -6,23 +6,26 @@
 // Arithmetic: ZGEQR2 order -- per column the reflector (ZLARFG: norm, IEEE
 // sqrt/div) and H_k^H = I - conj(tau_k) v_k v_k^H applied as a
 // matrix-vector product plus a rank-1 update (Table VI) -- in the
-// paper's 2D-cyclic register layout (Fig. 6): 8 row lanes x 4
-// column groups per warp, 6 warps = 24 column groups per CTA; element (r, c)
-// lives in lane (r mod 8, c mod 24), register (r div 8, c div 24).
+// paper's 2D-cyclic register layout (Fig. 6): a warp is one
+// column group (rows lane + 32 i, i < 8), 6 warps per CTA; element (r, c)
+// lives in lane r mod 32 of warp c mod 6, register (r div 32, c div 6).
 //
-// B200 design (see bqr_ll.cuh for the real 56 x 56 counterpart): the
+// B200 design (bqr_ll.cuh is the real 56 x 56 counterpart): the
 // right-looking class keeps the whole 240 x 67 tile in registers, one
-// matrix per SM, so 256 matrices take 1.73 rounds of a latency-bound
-// CTA.  Here the columns are factored in three blocks of 24, [0,24)
-// [24,48) [48,67): only the current block is in registers (30 rows x one
-// slot per lane); a block is loaded when it is reached, H_0..H_{c0-1} are
-// applied to it from shared memory (left-looking; no reflector chain), then
-// it is factored right-looking.  The 48 Householder vectors of the first two
-// blocks stay in shared memory (86 KB), so TWO matrices fit per SM (2 x 6
-// warps, 2 x 90 KB): 256 matrices are one resident round on 148 SMs.
+// matrix per SM, so 256 matrices take 1.73 rounds.  Here the columns are
+// factored in two blocks of 36, [0,36) and [36,67): only the current block
+// is in registers (8 rows x 6 slots per lane); block 1 is loaded when block
+// 0 is done, H_0..H_35 are applied to it from shared memory (left-looking,
+// no reflector chain), then it is factored right-looking.  The 36 vectors of
+// block 0 stay in shared memory (72 KB), block 1 publishes through a ring
+// of 9, so TWO matrices fit per SM (2 x 6 warps, 2 x 92 KB) and 256 are one
+// resident round.  Every reflector has a "full" mbarrier: a warp waits only
+// for the vector it is about to apply (no per-column CTA rendezvous); the
+// ring is never overwritten while read because warp w publishes every 6th
+// column and must have applied every earlier vector first (lag <= G + 2).
 // Packed FP32 (fma.rn.f32x2) on the (re, im) pair with v as the broadcast
-// scalar operand; vectors live in shared memory as 16-byte chunks of two
-// rows, chunk-major so the 8 row lanes read consecutive chunks.
+// scalar operand; vectors as 16-byte chunks of two rows, chunk-major so the
+// 32 lanes read 512 contiguous bytes.
 #pragma once
 #include "bqr_common.cuh"
 
@@ -39,25 +42,25 @@ struct Args {
 };
 
 constexpr int kM = 240, kN = 66;
-constexpr int R = 8, MR = 30;          // row lanes; rows rg + 8 i, i < 30
-constexpr int kWarps = 6, G = 4 * kWarps;  // 24 column groups
+constexpr int R = 32, MR = 8;          // rows lane + 32 i, i < 8 (rows >= 240 are zero)
+constexpr int kWarps = 6, G = kWarps;  // a warp is a column group
 constexpr int kThreads = 32 * kWarps;
-constexpr int NSMAX = 1;
-constexpr int kNB = 3;
-// column blocks [0,24) [24,48) [48,72): one slot (24 columns) per lane
-__host__ __device__ constexpr int blk_c0(int b) { return 24 * b; }
-__host__ __device__ constexpr int blk_ns(int) { return 1; }
-constexpr int kKeepP = 6;  // row panels (8 columns each) of block 0: reflectors 0..47 kept
-// 16-byte chunks (two rows) per row lane of a reflector of row panel P
-__host__ __device__ constexpr int chunks(int P) { return (MR - P + 1) / 2; }
-__host__ __device__ constexpr int voff(int P) { return P == 0 ? 0 : voff(P - 1) + 8 * R * chunks(P - 1); }
-constexpr int kVStore = voff(kKeepP);          // float4 units
-constexpr int kRingChunks = chunks(kKeepP);    // >= chunks of every later panel
-constexpr int kRingOff = kVStore;
-constexpr int kRingBuf = kRingChunks * R;
-constexpr int kTauOff = kRingOff + 2 * kRingBuf;  // float4 units; 72 float2 taus follow
-constexpr size_t kSmemBytes = (size_t)kTauOff * 16 + 72 * 8;
-static_assert(kSmemBytes * 2 <= 228 * 1024 - 2048, "two CTAs per SM");
+constexpr int NS = 6;                  // slots per lane: a block is 36 columns
+constexpr int kNB = 2;
+constexpr int kBW = G * NS;            // block width
+__host__ __device__ constexpr int blk_c0(int b) { return kBW * b; }
+constexpr int kKeep = kBW;             // reflectors of block 0, kept
+constexpr int kChunks = 4;             // 16-byte chunks (2 rows) per lane and vector
+constexpr int kVec = kChunks * R;      // float4 per vector (2 KB)
+constexpr int kRing = G + 3;           // ring depth for the reflectors of block 1
+constexpr int kRingOff = kKeep * kVec;
+constexpr int kTauOff = kRingOff + kRing * kVec;  // float4 units: 72 float2 taus
+constexpr int kBarOff = kTauOff + 36;             // float4 units: 72 mbarriers
+constexpr size_t kSmemBytes = (size_t)kBarOff * 16 + 72 * 8;
+static_assert(2 * (kSmemBytes + 1024) <= 228 * 1024, "two CTAs per SM");
+// first register row of the vectors of 6-column group S6 (its first column / 32)
+__host__ __device__ constexpr int row0(int S6) { return (G * S6) / R; }
+static_assert(row0((kN - 1) / G) <= 2 && row0(kKeep / G - 1) == 0, "chunk layout");
 
 __device__ __forceinline__ float4 lds128(const float4 *p) {
   float4 v;
@@ -65,244 +68,235 @@ __device__ __forceinline__ float4 lds128(const float4 *p) {
   asm volatile("ld.shared.v4.f32 {%0,%1,%2,%3}, [%4];" : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "r"(s));
   return v;
 }
-__device__ __forceinline__ void bsync() { asm volatile("bar.sync 0;" ::: "memory"); }
+__device__ __forceinline__ unsigned su32(const void *p) { return (unsigned)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ bool mbar_try(const unsigned long long *bar, unsigned parity) {
+  unsigned ok;
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2, %3;\n\t"
+      "selp.u32 %0, 1, 0, p;\n}"
+      : "=r"(ok)
+      : "r"(su32(bar)), "r"(parity), "r"(1000000u)
+      : "memory");
+  return ok != 0;
+}
+__device__ __forceinline__ void wsync() { asm volatile("bar.warp.sync -1;" ::: "memory"); }
 
 struct Ctx {
-  float4 *vs;    // vector store (float4 chunks)
-  float2 *taus;  // [72]
-  int rg, cg, lane, warp;
-  float2 *Ab;    // this lane's row rg of the matrix (column 0)
-  float2 *Bb;    // this lane's row rg of the right-hand side, or null
+  float4 *vs;
+  float2 *taus;
+  unsigned long long *full;  // [72]
+  unsigned parity;
+  int lane, warp;
+  float2 *Ab;  // this lane's row of column 0
+  float2 *Bb;  // this lane's row of the right-hand side, or null
   int lda;
 };
 
-using Tile = float2[MR][NSMAX];
+using Tile = float2[MR][NS];
 
-// this lane's chunk 0 of reflector k = 8P + kk (rows 8P + rg, 8P + 8 + rg, ...)
-template <int P>
-__device__ __forceinline__ float4 *vptr(const Ctx &c, int kk) {
-  if constexpr (P < kKeepP) {
-    return c.vs + voff(P) + kk * R * chunks(P) + c.rg;
-  } else {
-    return c.vs + kRingOff + (kk & 1) * kRingBuf + c.rg;
+__device__ __forceinline__ float4 *vptr(const Ctx &c, int k) {
+  return c.vs + (k < kKeep ? k * kVec : kRingOff + ((k - kKeep) % kRing) * kVec) + c.lane;
+}
+__device__ __forceinline__ void wait_full(const Ctx &c, int k) {
+  while (!mbar_try(c.full + k, c.parity)) {
   }
 }
-
 __device__ __forceinline__ float2 f2(float x, float y) { return make_float2(x, y); }
 
-// H_k^H on slots [J0, J1), rows from register row P (v zero above its pivot):
-// w = v^H a (reduced over the 8 row lanes), a -= v (conj(tau) w); MASK0: the
-// first slot only for columns cg > kkg (the pivot slot; kkg = pivot's group)
-template <int P, int J0, int J1, bool MASK0>
-__device__ __forceinline__ void apply(const Ctx &c, Tile &a, const float4 *vp, float2 ct, int kkg) {
+// H_k^H on slots [J0, J1) of this warp, rows from register row I0 (v is zero
+// above its pivot): w = v^H a (butterfly over the 32 lanes), a -= v conj(tau) w
+template <int I0, int J0, int J1>
+__device__ __forceinline__ void apply3(Tile &a, const float4 *vp, float2 ct) {
   if constexpr (J0 < J1) {
-    constexpr int NS = J1 - J0;
-    constexpr int NQ = chunks(P);
-    float2 wa[NS][2], wb[NS][2];
+    constexpr int N = J1 - J0;
+    float2 wa[N], wb[N];
 #pragma unroll
-    for (int j = 0; j < NS; ++j) wa[j][0] = wa[j][1] = wb[j][0] = wb[j][1] = f2(0.f, 0.f);
+    for (int j = 0; j < N; ++j) wa[j] = wb[j] = f2(0.f, 0.f);
 #pragma unroll
-    for (int q = 0; q < NQ; ++q) {
-      const float4 f = lds128(vp + q * R);
-      const int i = P + 2 * q;
+    for (int q = 0; q < kChunks; ++q) {
+      const int i = I0 + 2 * q;
+      if (i < MR) {
+        const float4 f = lds128(vp + q * R);
 #pragma unroll
-      for (int j = 0; j < NS; ++j) {
-        wa[j][0] = __ffma2_rn(f2(f.x, f.x), a[i][J0 + j], wa[j][0]);
-        wb[j][0] = __ffma2_rn(f2(f.y, f.y), a[i][J0 + j], wb[j][0]);
-        if (i + 1 < MR) {
-          wa[j][1] = __ffma2_rn(f2(f.z, f.z), a[i + 1][J0 + j], wa[j][1]);
-          wb[j][1] = __ffma2_rn(f2(f.w, f.w), a[i + 1][J0 + j], wb[j][1]);
+        for (int j = 0; j < N; ++j) {
+          wa[j] = __ffma2_rn(a[i][J0 + j], f2(f.x, f.x), wa[j]);
+          wb[j] = __ffma2_rn(a[i][J0 + j], f2(f.y, f.y), wb[j]);
+          if (i + 1 < MR) {
+            wa[j] = __ffma2_rn(a[i + 1][J0 + j], f2(f.z, f.z), wa[j]);
+            wb[j] = __ffma2_rn(a[i + 1][J0 + j], f2(f.w, f.w), wb[j]);
+          }
         }
       }
     }
-    float2 t[NS];
+    float2 t[N];
 #pragma unroll
-    for (int j = 0; j < NS; ++j) {
-      const float2 A2 = __fadd2_rn(wa[j][0], wa[j][1]), B2 = __fadd2_rn(wb[j][0], wb[j][1]);
-      float2 s = f2(A2.x + B2.y, A2.y - B2.x);  // conj(v)^T a
+    for (int j = 0; j < N; ++j) {
+      float2 s = f2(wa[j].x + wb[j].y, wa[j].y - wb[j].x);  // sum conj(v) a
 #pragma unroll
       for (int o = 1; o < R; o <<= 1)
         s = __fadd2_rn(s, f2(__shfl_xor_sync(0xffffffffu, s.x, o), __shfl_xor_sync(0xffffffffu, s.y, o)));
-      // t = conj(tau) * s
-      float2 tt = f2(fmaf(ct.x, s.x, -ct.y * s.y), fmaf(ct.x, s.y, ct.y * s.x));
-      if (MASK0 && j == 0) tt = c.cg > kkg ? tt : f2(0.f, 0.f);
-      t[j] = tt;
+      t[j] = f2(fmaf(ct.x, s.x, -ct.y * s.y), fmaf(ct.x, s.y, ct.y * s.x));
     }
 #pragma unroll
-    for (int q = 0; q < NQ; ++q) {
-      const float4 f = lds128(vp + q * R);
-      const int i = P + 2 * q;
+    for (int q = 0; q < kChunks; ++q) {
+      const int i = I0 + 2 * q;
+      if (i < MR) {
+        const float4 f = lds128(vp + q * R);
 #pragma unroll
-      for (int j = 0; j < NS; ++j) {
-        const float2 n1 = f2(-t[j].x, -t[j].y), n2 = f2(t[j].y, -t[j].x);
-        a[i][J0 + j] = __ffma2_rn(f2(f.y, f.y), n2, __ffma2_rn(f2(f.x, f.x), n1, a[i][J0 + j]));
-        if (i + 1 < MR)
-          a[i + 1][J0 + j] = __ffma2_rn(f2(f.w, f.w), n2, __ffma2_rn(f2(f.z, f.z), n1, a[i + 1][J0 + j]));
+        for (int j = 0; j < N; ++j) {
+          const float2 n1 = f2(-t[j].x, -t[j].y), n2 = f2(t[j].y, -t[j].x);
+          a[i][J0 + j] = __ffma2_rn(f2(f.y, f.y), n2, __ffma2_rn(f2(f.x, f.x), n1, a[i][J0 + j]));
+          if (i + 1 < MR)
+            a[i + 1][J0 + j] = __ffma2_rn(f2(f.w, f.w), n2, __ffma2_rn(f2(f.z, f.z), n1, a[i + 1][J0 + j]));
+        }
       }
     }
   }
 }
+// slots [J0, J1) in passes of at most three (bounds the live accumulators)
+template <int I0, int J0, int J1>
+__device__ __forceinline__ void apply(Tile &a, const float4 *vp, float2 ct) {
+  if constexpr (J0 < J1) {
+    constexpr int JM = J0 + 3 < J1 ? J0 + 3 : J1;
+    apply3<I0, J0, JM>(a, vp, ct);
+    apply<I0, JM, J1>(a, vp, ct);
+  }
+}
 
-// ZLARFG of column kn = 8 P + kr in slot S (owner lanes: cg == group of kn)
-template <int P, int S>
-__device__ __forceinline__ Reflector<float2> reflector(const Ctx &c, const Tile &a, int kr) {
-  float2 acc[2] = {f2(0.f, 0.f), f2(0.f, 0.f)};
+// ZLARFG of column kn held in slot S of this (owner) warp, rows from I0;
+// then the column becomes [R; V] and v_kn, tau_kn are published
+template <int I0, int S>
+__device__ __forceinline__ void reflect_publish(const Ctx &c, Tile &a, int kn) {
+  float2 acc = f2(0.f, 0.f);
   float2 alpha = f2(0.f, 0.f);
 #pragma unroll
-  for (int i = P; i < MR; ++i) {
+  for (int i = I0; i < MR; ++i) {
+    const int r = c.lane + R * i;
     float2 x = a[i][S];
-    if (i == P) {
-      alpha = c.rg == kr ? x : f2(0.f, 0.f);
-      x = c.rg > kr ? x : f2(0.f, 0.f);
-    }
-    acc[(i - P) & 1] = __ffma2_rn(x, x, acc[(i - P) & 1]);
+    alpha = r == kn ? x : alpha;
+    x = r > kn ? x : f2(0.f, 0.f);
+    acc = __ffma2_rn(x, x, acc);
   }
-  const float2 s2 = __fadd2_rn(acc[0], acc[1]);
-  float sig = s2.x + s2.y;
+  float sig = acc.x + acc.y;
 #pragma unroll
   for (int o = 1; o < R; o <<= 1) sig += __shfl_xor_sync(0xffffffffu, sig, o);
-  const int src = (c.lane & ~(R - 1)) | kr;
+  const int src = kn & (R - 1);
   alpha = f2(__shfl_sync(0xffffffffu, alpha.x, src), __shfl_sync(0xffffffffu, alpha.y, src));
-  return make_reflector(alpha, sig);
-}
-
-// owner lanes (cg == kg): v = x scal below the pivot, 1 at it, 0 above; the
-// column becomes [R; V] (beta at the pivot); v and tau go to shared memory
-template <int P, int S>
-__device__ __forceinline__ void publish(const Ctx &c, Tile &a, const Reflector<float2> &hh, int kr, int kg,
-                                        float4 *vdst, float2 *tslot) {
-  const bool own = c.cg == kg;
-  constexpr int NQ = chunks(P);
+  const Reflector<float2> h = make_reflector(alpha, sig);
+  float4 *vd = vptr(c, kn);
 #pragma unroll
-  for (int q = 0; q < NQ; ++q) {
+  for (int q = 0; q < kChunks; ++q) {
     float2 v[2];
 #pragma unroll
-    for (int h = 0; h < 2; ++h) {
-      const int i = P + 2 * q + h;
+    for (int e = 0; e < 2; ++e) {
+      const int i = I0 + 2 * q + e;
       if (i >= MR) {
-        v[h] = f2(0.f, 0.f);
+        v[e] = f2(0.f, 0.f);
         continue;
       }
+      const int r = c.lane + R * i;
       const float2 x = a[i][S];
-      const float2 xs = f2(fmaf(x.x, hh.scal.x, -x.y * hh.scal.y), fmaf(x.x, hh.scal.y, x.y * hh.scal.x));
-      if (i == P) {
-        v[h] = c.rg > kr ? xs : (c.rg == kr ? f2(1.f, 0.f) : f2(0.f, 0.f));
-        if (own) a[i][S] = c.rg > kr ? xs : (c.rg == kr ? f2(hh.beta, 0.f) : x);
-      } else {
-        v[h] = xs;
-        if (own) a[i][S] = xs;
-      }
+      const float2 xs = f2(fmaf(x.x, h.scal.x, -x.y * h.scal.y), fmaf(x.x, h.scal.y, x.y * h.scal.x));
+      v[e] = r > kn ? xs : (r == kn ? f2(1.f, 0.f) : f2(0.f, 0.f));
+      a[i][S] = r > kn ? xs : (r == kn ? f2(h.beta, 0.f) : x);
     }
-    if (own) vdst[q * R] = make_float4(v[0].x, v[0].y, v[1].x, v[1].y);
+    vd[q * R] = make_float4(v[0].x, v[0].y, v[1].x, v[1].y);
   }
-  if (own && c.rg == 0) *tslot = hh.tau;
+  if (c.lane == 0) c.taus[kn] = h.tau;
+  wsync();  // lane 0's tau store before every lane's release
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(su32(c.full + kn)) : "memory");
 }
 
 // ---------------------------------------------------------------- phases
-template <int B, int J>
-__device__ __forceinline__ void load_slot(const Ctx &c, Tile &a) {
-  if constexpr (J < blk_ns(B)) {
-    const int col = blk_c0(B) + c.cg + G * J;
-    const float2 *p = col < kN ? c.Ab + (long long)col * c.lda : c.Bb;
+template <int B>
+__device__ __forceinline__ void load_block(const Ctx &c, Tile &a) {
+#pragma unroll
+  for (int j = 0; j < NS; ++j) {
+    const int col = blk_c0(B) + c.warp + G * j;
     const bool live = col < kN || (col == kN && c.Bb != nullptr);
+    const float2 *p = col < kN ? c.Ab + (long long)col * c.lda : c.Bb;
 #pragma unroll
-    for (int i = 0; i < MR; ++i) a[i][J] = live ? p[8 * i] : f2(0.f, 0.f);
+    for (int i = 0; i < MR; ++i) a[i][j] = (live && c.lane + R * i < kM) ? p[R * i] : f2(0.f, 0.f);
   }
 }
-template <int B, int J>
-__device__ __forceinline__ void store_slot(const Ctx &c, const Tile &a) {
-  if constexpr (J < blk_ns(B)) {
-    const int col = blk_c0(B) + c.cg + G * J;
+template <int B>
+__device__ __forceinline__ void store_block(const Ctx &c, const Tile &a) {
+#pragma unroll
+  for (int j = 0; j < NS; ++j) {
+    const int col = blk_c0(B) + c.warp + G * j;
+    const bool live = col < kN || (col == kN && c.Bb != nullptr);
     float2 *p = col < kN ? c.Ab + (long long)col * c.lda : c.Bb;
-    if (col < kN || (col == kN && c.Bb != nullptr)) {
 #pragma unroll
-      for (int i = 0; i < MR; ++i) p[8 * i] = a[i][J];
-    }
+    for (int i = 0; i < MR; ++i)
+      if (live && c.lane + R * i < kM) p[R * i] = a[i][j];
   }
 }
 
-// left-looking: H_0 .. H_{c0-1} (row panels 0 .. c0/8 - 1) on block B
-template <int B, int P>
+// left-looking: H_0 .. H_{c0-1} (vectors from register row 0) on every slot
+template <int B>
 __device__ __forceinline__ void left(const Ctx &c, Tile &a) {
-  if constexpr (P < blk_c0(B) / 8) {
-#pragma unroll 2
-    for (int kk = 0; kk < 8; ++kk) {
-      const float2 tau = c.taus[8 * P + kk];
-      apply<P, 0, blk_ns(B), false>(c, a, vptr<P>(c, kk), f2(tau.x, -tau.y), 0);
-    }
-    left<B, P + 1>(c, a);
+#pragma unroll 1
+  for (int k = 0; k < blk_c0(B); ++k) {
+    wait_full(c, k);
+    const float2 tau = c.taus[k];
+    apply<0, 0, NS>(a, vptr(c, k), f2(tau.x, -tau.y));
   }
 }
 
-// right-looking factorisation of block B, row panel P (columns 8P .. 8P+7,
-// slot s = (8P - c0) / 24); reflector 8P is published on entry.  Step k:
-// the warp owning column k+1 applies H_k to that slot first, forms and
-// publishes reflector k+1, then applies H_k to the rest; other warps apply
-// H_k to their live slots; one CTA barrier per column.
-template <int B, int P>
+// right-looking factorisation of block B, slot S (columns c0 + 6S + w):
+// step k = c0 + 6S + kk waits for v_k; the owner of column k+1 applies H_k
+// to the slot holding it, publishes reflector k+1, then applies H_k to its
+// other live slots; every other warp applies H_k to its live slots (its
+// slot S only if its column there is > k)
+template <int B, int S>
 __device__ __forceinline__ void panels(const Ctx &c, Tile &a) {
-  constexpr int c0 = blk_c0(B), NS = blk_ns(B);
-  constexpr int P0 = c0 / 8, PE = (c0 + G * NS) / 8;
-  if constexpr (P < PE && 8 * P < kN) {
-    constexpr int s = (8 * P - c0) / G;
-    constexpr int kg0 = (8 * P - c0) % G;  // group of column 8P
-    constexpr int kend = (8 * P + 8 < kN ? 8 * P + 8 : kN) - 8 * P;
+  if constexpr (S < NS) {
+    constexpr int c0 = blk_c0(B), S6 = (c0 / G) + S, I0 = row0(S6);
+    constexpr int kbeg = c0 + G * S;
+    constexpr int kend = kbeg + G < kN ? kbeg + G : kN;
 #pragma unroll 1
-    for (int kk = 0; kk < kend; ++kk) {
-      bsync();
-      const int k = 8 * P + kk;
+    for (int k = kbeg; k < kend; ++k) {
+      const int kk = k - kbeg;
+      wait_full(c, k);
       const float2 tau = c.taus[k];
       const float2 ct = f2(tau.x, -tau.y);
-      const float4 *vp = vptr<P>(c, kk);
+      const float4 *vp = vptr(c, k);
       const int kn = k + 1;
-      if (kk + 1 < 8) {
-        // column k+1 in this panel and slot
-        const int kgn = kg0 + kk + 1;
-        if (kn < kN && c.warp == kgn / 4) {
-          apply<P, s, s + 1, true>(c, a, vp, ct, kg0 + kk);
-          const Reflector<float2> h = reflector<P, s>(c, a, kk + 1);
-          publish<P, s>(c, a, h, kk + 1, kgn, vptr<P>(c, kk + 1), c.taus + kn);
-          apply<P, s + 1, NS, false>(c, a, vp, ct, 0);
+      if (kk + 1 < G) {
+        if (kn < kN && c.warp == kk + 1) {
+          apply<I0, S, S + 1>(a, vp, ct);
+          reflect_publish<I0, S>(c, a, kn);
+          apply<I0, S + 1, NS>(a, vp, ct);
+        } else if (c.warp > kk) {
+          apply<I0, S, NS>(a, vp, ct);
         } else {
-          // a warp whose four column groups are all factored (<= the
-          // pivot's group) has nothing left in this block's slot
-          if (4 * c.warp + 3 > kg0 + kk) apply<P, s, NS, true>(c, a, vp, ct, kg0 + kk);
+          apply<I0, S + 1, NS>(a, vp, ct);
         }
       } else {
-        // column k+1 opens row panel P+1 (maybe the next slot)
-        constexpr int sn = (8 * P + 8 - c0) / G, kgn = (8 * P + 8 - c0) % G;
-        if (kn < kN && sn < NS && c.warp == kgn / 4) {
-          if constexpr (sn < NS) {
-            apply<P, s, s + 1, true>(c, a, vp, ct, kg0 + kk);
-            if constexpr (sn != s) apply<P, sn, sn + 1, false>(c, a, vp, ct, 0);
-            const Reflector<float2> h = reflector<P + 1, sn>(c, a, 0);
-            publish<P + 1, sn>(c, a, h, 0, kgn, vptr<P + 1>(c, 0), c.taus + kn);
-            apply<P, sn + 1, NS, false>(c, a, vp, ct, 0);
+        // column k+1 opens slot S+1 (owner: warp 0), unless the block ends
+        if constexpr (S + 1 < NS) {
+          if (kn < kN && c.warp == 0) {
+            apply<I0, S + 1, S + 2>(a, vp, ct);
+            reflect_publish<row0(S6 + 1), S + 1>(c, a, kn);
+            apply<I0, S + 2, NS>(a, vp, ct);
+          } else {
+            apply<I0, S + 1, NS>(a, vp, ct);
           }
-        } else {
-          // a warp whose four column groups are all factored (<= the
-          // pivot's group) has nothing left in this block's slot
-          if (4 * c.warp + 3 > kg0 + kk) apply<P, s, NS, true>(c, a, vp, ct, kg0 + kk);
         }
       }
     }
-    panels<B, P + 1>(c, a);
+    panels<B, S + 1>(c, a);
   }
 }
 
 template <int B>
 __device__ __forceinline__ void do_block(const Ctx &c, Tile &a) {
-  constexpr int P0 = blk_c0(B) / 8;
-  load_slot<B, 0>(c, a);
-  left<B, 0>(c, a);
-  // head reflector of the block (column c0: slot 0, group 0)
-  if (c.warp == 0) {
-    const Reflector<float2> h = reflector<P0, 0>(c, a, 0);
-    publish<P0, 0>(c, a, h, 0, 0, vptr<P0>(c, 0), c.taus + 8 * P0);
-  }
-  panels<B, P0>(c, a);
-  store_slot<B, 0>(c, a);
-  bsync();
+  load_block<B>(c, a);
+  left<B>(c, a);
+  if (c.warp == 0) reflect_publish<row0(blk_c0(B) / G), 0>(c, a, blk_c0(B));
+  panels<B, 0>(c, a);
+  store_block<B>(c, a);
 }
 
 __global__ void __launch_bounds__(kThreads, 2) geqrf_llc240_kernel(Args args) {
@@ -311,22 +305,28 @@ __global__ void __launch_bounds__(kThreads, 2) geqrf_llc240_kernel(Args args) {
   Ctx c;
   c.lane = t & 31;
   c.warp = __shfl_sync(0xffffffffu, t >> 5, 0);
-  c.rg = c.lane & (R - 1);
-  c.cg = 4 * c.warp + (c.lane >> 3);
   c.vs = smem_llc;
   c.taus = reinterpret_cast<float2 *>(smem_llc + kTauOff);
+  c.full = reinterpret_cast<unsigned long long *>(smem_llc + kBarOff);
   c.lda = args.lda;
+  if (t < kN) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(su32(c.full + t)), "r"(32) : "memory");
+  }
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  __syncthreads();
+  c.parity = 0;
 #pragma unroll 1
   for (long long mat = blockIdx.x; mat < args.batch; mat += gridDim.x) {
-    c.Ab = args.A + mat * args.strideA + c.rg;
-    c.Bb = args.nrhs > 0 ? args.B + mat * args.strideB + c.rg : nullptr;
+    c.Ab = args.A + mat * args.strideA + c.lane;
+    c.Bb = args.nrhs > 0 ? args.B + mat * args.strideB + c.lane : nullptr;
     Tile a;
     do_block<0>(c, a);
     do_block<1>(c, a);
-    do_block<2>(c, a);
+    __syncthreads();  // every vector consumed, every tau published
     float2 *tg = args.tau + mat * args.strideT;
     for (int i = t; i < kN; i += kThreads) tg[i] = c.taus[i];
-    bsync();
+    __syncthreads();
+    c.parity ^= 1u;
   }
 }
 
