@@ -62,6 +62,8 @@ rows = list(csv.reader(io.TextIOWrapper(op(csvp, "rb"))))
 hdr = rows[1]
 ix = {h: i for i, h in enumerate(hdr)}
 base = int(rows[2][ix["Address"]], 16)
+stc = [h for h in hdr if h.startswith("stall_") and "Not Issued" not in h]
+reasons = defaultdict(lambda: defaultdict(int))
 incl = defaultdict(lambda: [0, 0])
 self_ = defaultdict(lambda: [0, 0])
 tot = [0, 0]
@@ -87,6 +89,8 @@ for r in rows[2:]:
     for nm in names:
         incl[nm][0] += ex
         incl[nm][1] += sm
+        for h in stc:
+            reasons[nm][h[6:]] += int(r[ix[h]] or 0)
     # outer call line (caller context)
     outer = [ln for f, ln in ch if f.endswith(srcp.split("/")[-1])]
     if outer:
@@ -95,6 +99,11 @@ print(f"total executed {tot[0]}  samples {tot[1]}")
 print("%-22s %12s %7s %8s %7s" % ("function (inclusive)", "exec", "exec%", "samples", "samp%"))
 for k, (e, s) in sorted(incl.items(), key=lambda kv: -kv[1][1]):
     print("%-22s %12d %6.1f%% %8d %6.1f%%" % (k, e, 100 * e / tot[0], s, 100 * s / max(1, tot[1])))
+print("stall reasons (inclusive):")
+for k, (e, s_) in sorted(incl.items(), key=lambda kv: -kv[1][1]):
+    rs = reasons[k]
+    tot_r = max(1, sum(rs.values()))
+    print("  %-20s " % k + " ".join(f"{n}={100 * v / tot_r:.0f}%" for n, v in sorted(rs.items(), key=lambda kv: -kv[1])[:7]))
 print("%-22s %12s %7s %8s %7s" % ("function (self)", "exec", "exec%", "samples", "samp%"))
 for k, (e, s) in sorted(self_.items(), key=lambda kv: -kv[1][1]):
     print("%-22s %12d %6.1f%% %8d %6.1f%%" % (k, e, 100 * e / tot[0], s, 100 * s / max(1, tot[1])))
