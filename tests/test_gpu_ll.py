@@ -1,0 +1,75 @@
+"""GPU parity of the round-2 left-looking C3 class (csrc/bqr_ll.cuh,
+`ll_f32_56x56_left4_x2`) on the paths the bench shape does not take: the
+persistent warp loop (more pairs than one resident round), odd batches (the
+spare half-warp), even lda > m (row-pair loads into padded storage), and the
+fallbacks to the right-looking class (odd lda, 4-byte-aligned base).
+Comparator: oracle/compare.py (north-star tolerances, reading Q10)."""
+import ctypes
+
+import numpy as np
+import pytest
+
+import bqr_inputs
+from oracle.compare import compare_geqrf
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+if not torch.cuda.is_available():  # pragma: no cover
+    pytest.skip("needs a GPU", allow_module_level=True)
+
+import paper_conf_ipps_andersonsk12_b200 as bqr  # noqa: E402
+from gpu_util import geqrf_gpu  # noqa: E402
+
+
+def test_dispatch_is_left_looking():
+    assert bqr.kernel_name(bqr.R32, 56, 56) == "ll_f32_56x56_left4_x2"
+
+
+def test_persistent_loop_second_pass():
+    """5,100 matrices = 2,550 pairs on <= 148 CTAs of 17 warps: chunk 18, so
+    warp 0 of every CTA factors a second pair (matrices 36 b + 34, 36 b + 35)
+    after its first; those and a sample of the rest against the oracle."""
+    batch = 5100
+    A = bqr_inputs.random_batch(56, 56, batch, "f32", seed=5100)
+    out, tau = geqrf_gpu(A, 56)
+    second = [i for b in range(0, 148, 5) for i in (36 * b + 34, 36 * b + 35) if i < batch]
+    idx = sorted(set(second) | set(range(0, batch, 97)) | {batch - 1})
+    rep = compare_geqrf(A[idx], 56, out[idx], tau[idx])
+    assert rep["ok"], rep
+
+
+@pytest.mark.parametrize("batch", [1, 2, 3, 33, 149, 297])
+def test_odd_and_small_batches(batch):
+    A = bqr_inputs.random_batch(56, 56, batch, "f32", seed=700 + batch)
+    out, tau = geqrf_gpu(A, 56)
+    rep = compare_geqrf(A, 56, out, tau)
+    assert rep["ok"], rep
+
+
+@pytest.mark.parametrize("lda", [58, 64, 57])
+def test_lda_padding(lda):
+    """even lda: the left-looking class (8-byte row-pair accesses); odd lda:
+    the right-looking class of the same shape.  NaN sentinels in the padding
+    rows must survive untouched."""
+    A = bqr_inputs.random_batch(56, 56, 71, "f32", seed=lda, lda=lda)
+    out, tau = geqrf_gpu(A, 56)
+    rep = compare_geqrf(A, 56, out, tau)
+    assert rep["ok"] and rep["padding_ok"], rep
+
+
+def test_four_byte_aligned_base():
+    """A base that is 4- but not 8-byte aligned takes the right-looking class."""
+    batch = 40
+    A = bqr_inputs.random_batch(56, 56, batch, "f32", seed=77)
+    flat = torch.zeros(A.size + 1, dtype=torch.float32, device="cuda")
+    flat[1:] = torch.from_numpy(np.ascontiguousarray(A).reshape(-1)).cuda()
+    tau = torch.empty((batch, 56), dtype=torch.float32, device="cuda")
+    st = bqr.load().bqr_geqrf_batched(bqr.R32, 56, 56, batch, ctypes.c_void_p(flat.data_ptr() + 4), 56,
+                                      ctypes.c_void_p(tau.data_ptr()),
+                                      ctypes.c_void_p(torch.cuda.current_stream().cuda_stream))
+    assert st == 0
+    torch.cuda.synchronize()
+    out = flat[1:].cpu().numpy().reshape(A.shape)
+    rep = compare_geqrf(A, 56, out, tau.cpu().numpy())
+    assert rep["ok"], rep

@@ -117,7 +117,8 @@ CASES = [
     (case_geqrf, ("f32", 4, 4, 300)),          # tiny, thread per matrix
     (case_geqrf, ("c64", 8, 8, 100)),
     (case_geqrf, ("f32", 16, 16, 64)),         # sub-warp staged groups
-    (case_geqrf, ("f32", 56, 56, 2400)),       # C3 class: persistent warp loop, > 1 pair per warp
+    (case_geqrf, ("f32", 56, 56, 5100)),       # C3 left-looking class: > 17 pairs on some CTAs (warp loop)
+    (case_geqrf, ("f32", 56, 56, 33)),         # odd batch: the spare half-warp repeats its neighbour
     (case_geqrf, ("f32", 33, 30, 40)),
     (case_geqrf, ("c64", 32, 32, 40)),         # warp groups
     (case_geqrf, ("f32", 80, 80, 20)),         # CTA groups, named barriers
@@ -140,7 +141,12 @@ CASES = [
     (case_host, ("f32", 56, 56, 300)),
 ]
 if QUICK:
-    CASES = [c for i, c in enumerate(CASES) if i in (0, 3, 6, 8, 12, 13, 14, 18, 20, 23)]
+    CASES = [c for i, c in enumerate(CASES) if i in (0, 3, 4, 7, 9, 13, 14, 15, 19, 21, 24)]
+if "--new" in sys.argv:
+    # this session's kernels only: the left-looking C3 class, and (run with
+    # BQR_FORCE_VARIANT=alt_llc_c64_240x66_left3[_aug]) the C4 experiment
+    CASES = [(case_geqrf, ("f32", 56, 56, 5100)), (case_geqrf, ("f32", 56, 56, 33)),
+             (case_geqrf, ("c64", 240, 66, 300)), (case_qhb_gels, ("c64", 240, 66, 300))]
 
 for fn, args in CASES:
     print("ok", fn(*args), flush=True)
