@@ -95,6 +95,12 @@ struct Ctx {
 
 using Tile = float2[MR][NS];
 
+// lazy rest-update of the next-but-one owner: parity green but slower on
+// B200 (134 vs 119 us; a lone matrix 119.6 vs 113 us), off
+#ifndef BQR_LLC_LAZY
+#define BQR_LLC_LAZY 0
+#endif
+
 __device__ __forceinline__ float4 *vptr(const Ctx &c, int k) {
   return c.vs + (k < kKeep ? k * kVec : kRingOff + ((k - kKeep) % kRing) * kVec) + c.lane;
 }
@@ -253,8 +259,10 @@ template <int B, int S>
 __device__ __forceinline__ void panels(const Ctx &c, Tile &a) {
   if constexpr (S < NS) {
     constexpr int c0 = blk_c0(B), S6 = (c0 / G) + S, I0 = row0(S6);
+    constexpr int I0p = S > 0 ? row0(S6 - 1) : I0;  // rows of the previous slot's vectors
     constexpr int kbeg = c0 + G * S;
     constexpr int kend = kbeg + G < kN ? kbeg + G : kN;
+    constexpr int klim = c0 + kBW < kN ? c0 + kBW : kN;  // pivots of this block: k < klim
 #pragma unroll 1
     for (int k = kbeg; k < kend; ++k) {
       const int kk = k - kbeg;
@@ -262,7 +270,46 @@ __device__ __forceinline__ void panels(const Ctx &c, Tile &a) {
       const float2 tau = c.taus[k];
       const float2 ct = f2(tau.x, -tau.y);
       const float4 *vp = vptr(c, k);
-      const int kn = k + 1;
+      const int kn = k + 1, kn2 = k + 2;
+#if BQR_LLC_LAZY
+      // lazy rest-update (the right-looking class's LAZY scheme): the owner of
+      // column k+2 applies H_k only to the slot holding k+2 and defers its
+      // other slots to step k+1, after it has published v_{k+2}; otherwise
+      // that rest-update sits between v_{k+1} arriving and its own chain
+      const bool o1 = kn < klim && c.warp == (kk + 1) % G;
+      const bool o2 = !o1 && kn2 < klim && c.warp == (kk + 2) % G;
+      if (o1) {
+        const float2 tp = k > c0 ? c.taus[k - 1] : f2(0.f, 0.f);
+        const float2 ctp = f2(tp.x, -tp.y);
+        const float4 *vpp = vptr(c, k > c0 ? k - 1 : k);
+        if (kk + 1 < G) {
+          apply<I0, S, S + 1>(a, vp, ct);
+          reflect_publish<I0, S>(c, a, kn);
+          if (k > c0) {
+            if (kk == 0)
+              apply<I0p, S + 1, NS>(a, vpp, ctp);
+            else
+              apply<I0, S + 1, NS>(a, vpp, ctp);
+          }
+          apply<I0, S + 1, NS>(a, vp, ct);
+        } else if constexpr (S + 1 < NS) {
+          apply<I0, S + 1, S + 2>(a, vp, ct);
+          reflect_publish<row0(S6 + 1), S + 1>(c, a, kn);
+          if (k > c0) apply<I0, S + 2, NS>(a, vpp, ctp);
+          apply<I0, S + 2, NS>(a, vp, ct);
+        }
+      } else if (o2) {
+        if (kk + 2 < G) {
+          apply<I0, S, S + 1>(a, vp, ct);
+        } else {
+          apply<I0, S + 1, S + 2>(a, vp, ct);
+        }
+      } else if (c.warp > kk) {
+        apply<I0, S, NS>(a, vp, ct);
+      } else {
+        apply<I0, S + 1, NS>(a, vp, ct);
+      }
+#else
       if (kk + 1 < G) {
         if (kn < kN && c.warp == kk + 1) {
           apply<I0, S, S + 1>(a, vp, ct);
@@ -285,6 +332,7 @@ __device__ __forceinline__ void panels(const Ctx &c, Tile &a) {
           }
         }
       }
+#endif
     }
     panels<B, S + 1>(c, a);
   }
