@@ -82,6 +82,21 @@ __device__ __forceinline__ bool mbar_try(const unsigned long long *bar, unsigned
 }
 __device__ __forceinline__ void wsync() { asm volatile("bar.warp.sync -1;" ::: "memory"); }
 
+#ifdef BQR_LLC_TIMING
+// debug builds only: clock64 of CTA 0's first matrix, [warp][k][0] = wait for
+// v_k returned, [warp][k][1] = v_{k+1} published (its owner), [warp][70..72]
+// = block 0 start, block 1 start (before its loads), after block 1's left
+static __device__ unsigned long long g_llc_dbg[kWarps * 74 * 2];
+#define LLC_STAMP(c, k, e)                                                                   \
+  do {                                                                                        \
+    if (blockIdx.x == 0 && (c).lane == 0 && (c).first) g_llc_dbg[((c).warp * 74 + (k)) * 2 + (e)] = clock64(); \
+  } while (0)
+#else
+#define LLC_STAMP(c, k, e) \
+  do {                     \
+  } while (0)
+#endif
+
 struct Ctx {
   float4 *vs;
   float2 *taus;
@@ -91,6 +106,9 @@ struct Ctx {
   float2 *Ab;  // this lane's row of column 0
   float2 *Bb;  // this lane's row of the right-hand side, or null
   int lda;
+#ifdef BQR_LLC_TIMING
+  bool first;
+#endif
 };
 
 using Tile = float2[MR][NS];
@@ -210,6 +228,7 @@ __device__ __forceinline__ void reflect_publish(const Ctx &c, Tile &a, int kn) {
     vd[q * R] = make_float4(v[0].x, v[0].y, v[1].x, v[1].y);
   }
   if (c.lane == 0) c.taus[kn] = h.tau;
+  LLC_STAMP(c, kn, 1);
   wsync();  // lane 0's tau store before every lane's release
   asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(su32(c.full + kn)) : "memory");
 }
@@ -267,6 +286,7 @@ __device__ __forceinline__ void panels(const Ctx &c, Tile &a) {
     for (int k = kbeg; k < kend; ++k) {
       const int kk = k - kbeg;
       wait_full(c, k);
+      LLC_STAMP(c, k, 0);
       const float2 tau = c.taus[k];
       const float2 ct = f2(tau.x, -tau.y);
       const float4 *vp = vptr(c, k);
@@ -340,8 +360,10 @@ __device__ __forceinline__ void panels(const Ctx &c, Tile &a) {
 
 template <int B>
 __device__ __forceinline__ void do_block(const Ctx &c, Tile &a) {
+  LLC_STAMP(c, 70 + B, 0);
   load_block<B>(c, a);
   left<B>(c, a);
+  LLC_STAMP(c, 72 + B, 0);
   if (c.warp == 0) reflect_publish<row0(blk_c0(B) / G), 0>(c, a, blk_c0(B));
   panels<B, 0>(c, a);
   store_block<B>(c, a);
@@ -363,6 +385,9 @@ __global__ void __launch_bounds__(kThreads, 2) geqrf_llc240_kernel(Args args) {
   asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   __syncthreads();
   c.parity = 0;
+#ifdef BQR_LLC_TIMING
+  c.first = true;
+#endif
 #pragma unroll 1
   for (long long mat = blockIdx.x; mat < args.batch; mat += gridDim.x) {
     c.Ab = args.A + mat * args.strideA + c.lane;
@@ -375,6 +400,9 @@ __global__ void __launch_bounds__(kThreads, 2) geqrf_llc240_kernel(Args args) {
     for (int i = t; i < kN; i += kThreads) tg[i] = c.taus[i];
     __syncthreads();
     c.parity ^= 1u;
+#ifdef BQR_LLC_TIMING
+    c.first = false;
+#endif
   }
 }
 
