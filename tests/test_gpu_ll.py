@@ -73,3 +73,51 @@ def test_four_byte_aligned_base():
     out = flat[1:].cpu().numpy().reshape(A.shape)
     rep = compare_geqrf(A, 56, out, tau.cpu().numpy())
     assert rep["ok"], rep
+
+
+# ------------------------------------------------------------ left-looking LU (bqr_lll.cuh)
+def _lu_gpu(A_cm, m):
+    batch, n, lda = A_cm.shape
+    buf = torch.from_numpy(np.ascontiguousarray(A_cm)).cuda()
+    info = torch.full((batch,), -7, dtype=torch.int32, device="cuda")
+    st = bqr.load().bqr_getrf_np_batched(bqr.R32, m, n, batch, ctypes.c_void_p(buf.data_ptr()), lda,
+                                         ctypes.c_void_p(info.data_ptr()), None)
+    assert st == 0, st
+    torch.cuda.synchronize()
+    return buf.cpu().numpy(), info.cpu().numpy()
+
+
+def test_lu56_zero_pivot_info():
+    """Row 30 zero left of and on the diagonal: l_30,j = 0 for j < 30, so
+    u_30,30 = a_30,30 = 0 exactly -> scale 0, info = 31, the elimination goes
+    on (reading L1); matrix 0 also has a zero first pivot (info 1)."""
+    from oracle.compare import compare_lu
+    A = bqr_inputs.diag_dominant_batch(56, 5, "f32", seed=56)  # storage (batch, col, row)
+    A[1, :31, 30] = 0.0
+    A[0, 0, :] = 0.0
+    out, info = _lu_gpu(A, 56)
+    assert list(info[:2]) == [1, 31] and list(info[2:]) == [0, 0, 0]
+    rep = compare_lu(A, 56, out, info)
+    assert rep["ok"], rep
+
+
+@pytest.mark.parametrize("lda", [58, 57])
+def test_lu56_lda_padding(lda):
+    from oracle.compare import compare_lu
+    A = bqr_inputs.diag_dominant_batch(56, 35, "f32", seed=lda, lda=lda)
+    out, info = _lu_gpu(A, 56)
+    assert np.isnan(out[:, :, 56:]).all()
+    rep = compare_lu(A, 56, out, info)
+    assert rep["ok"], rep
+
+
+@pytest.mark.parametrize("batch", [1, 3, 10067])
+def test_lu56_batches(batch):
+    """odd batches (spare half-warp) and a batch whose CTAs factor up to
+    three pairs per warp (persistent loop), sampled against the oracle"""
+    from oracle.compare import compare_lu
+    A = bqr_inputs.diag_dominant_batch(56, batch, "f32", seed=900 + batch)
+    out, info = _lu_gpu(A, 56)
+    idx = sorted(set(range(0, batch, 53)) | {batch - 1})
+    rep = compare_lu(A[idx], 56, out[idx], info[idx])
+    assert rep["ok"], rep
