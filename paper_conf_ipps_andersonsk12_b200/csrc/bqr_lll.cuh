@@ -162,7 +162,9 @@ __device__ __forceinline__ void panels(Ctx &c, Tile &a) {
       }
       wsync();
       lapply<P, s, NS, true>(c, a, lp, kk);
-      wsync();  // the ring buffer of l is rewritten two steps later
+      // the two-entry ring (columns >= 40) is rewritten two steps later;
+      // the kept columns are never rewritten
+      if constexpr (P >= kKeepP) wsync();
     }
     store_slot<B, s>(c, a);
     load_slot<B + 1, s>(c, a);

@@ -1,3 +1,14 @@
-# L56 / GJ56 parity + timing (tools/lu_time.py) with the left-looking LU on and off
-python -m pytest tests/test_gpu_lu.py -q -p no:cacheprovider 2>&1 | tail -3 > gpurun_out/pt_lu.txt
-python bench.py --config L56 --no-also --no-c5 --no-cpu --steps 50 > gpurun_out/bench_l56.json 2> gpurun_out/bench_l56.err
+# L56 timing of experiment builds (BQR lib override) + parity of the LU tests
+for lib in "$@"; do
+python - "$lib" <<'PY'
+import sys, os, json
+sys.path.insert(0, os.getcwd())
+import paper_conf_ipps_andersonsk12_b200 as bqr
+bqr._LIB_PATH = os.path.abspath(sys.argv[1])
+import torch, bench
+w = bench.Workload("L56", 0, 1, torch, bqr)
+flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
+_, q = bench.time_workload(w, 50, 5, torch, None, 1, flush)
+print(json.dumps({"lib": sys.argv[1], "L56_us": round(q * 1e3, 2)}))
+PY
+done
