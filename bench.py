@@ -305,7 +305,7 @@ def roofline_obj(w: Workload, qr_ms: float, peaks: dict, n_sm: int, fused: bool 
     nbytes = w.bytes + (w.bytes_apply if fused else 0)
     t_roof, bound = bm.roofline_time_s(flops, nbytes, hbm, fp32)
     t = qr_ms / 1e3
-    kname = ({"lu": "lu_rf_kernel (LU, no pivoting)", "gj": "lu_rf_kernel (Gauss-Jordan)"}[w.kind]
+    kname = (w.bqr.load().bqr_lu_kernel_name(w.code, w.m, w.n, w.nrhs, int(w.kind == "gj")).decode()
              if w.kind != "qr" else
              w.bqr.load().bqr_qhb_kernel_name(w.code, w.m, w.n, w.nrhs).decode() if fused
              else w.bqr.kernel_name(w.code, w.m, w.n))

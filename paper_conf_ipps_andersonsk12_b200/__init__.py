@@ -68,6 +68,9 @@ def load():
         lib.bqr_getrf_np_batched.restype = i
         lib.bqr_gauss_jordan_batched.argtypes = [i, i, i, i, p, i, p, i, p, p]
         lib.bqr_gauss_jordan_batched.restype = i
+    if hasattr(lib, "bqr_lu_kernel_name"):
+        lib.bqr_lu_kernel_name.argtypes = [i, i, i, i, i]
+        lib.bqr_lu_kernel_name.restype = ctypes.c_char_p
     lib.bqr_geqrf_batched_host.argtypes = [i, i, i, i, p, i, p, p, sz, p]
     lib.bqr_host_workspace_bytes.argtypes = [i, i, i, i, i]
     lib.bqr_host_workspace_bytes.restype = sz
