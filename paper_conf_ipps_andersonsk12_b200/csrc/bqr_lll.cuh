@@ -126,49 +126,77 @@ __device__ __forceinline__ void left(const Ctx &c, Tile &a) {
   }
 }
 
-// elimination of block B, panel P (columns 4P .. 4P + 3 in slot s)
+// IEEE reciprocal of the pivot of column kn = 4 PP + kkn (slot S; row kn
+// in pair PP/2 of the lane rg = kr/2 of column group kkn), 0 for an exactly
+// zero pivot (info = kn + 1 of the first one; reading L1)
+template <int PP, int S>
+__device__ __forceinline__ float pivot_scale(Ctx &c, const Tile &a, int kkn, int kn) {
+  constexpr int q = PP / 2;
+  const int kr = 4 * (PP % 2) + kkn;
+  const float px = (kr & 1) ? a[q][S].y : a[q][S].x;
+  const float piv = __shfl_sync(0xffffffffu, px, (c.lane & 16) | (kkn * 4) | (kr >> 1));
+  const bool z = piv == 0.f;
+  c.info = (c.info == 0 && z) ? kn + 1 : c.info;
+  return z ? 0.f : __fdiv_rn(1.0f, piv);
+}
+
+// column k = 4P + kk (slot s): l = a * scale below the pivot, in place and
+// to shared memory (owner column group)
+template <int P, int S>
+__device__ __forceinline__ void publish_l(const Ctx &c, Tile &a, int kk, float scale, float *lp) {
+  constexpr int q0 = P / 2;
+  const int k = 4 * P + kk;
+  const bool own = c.cg == kk;
+#pragma unroll
+  for (int p = q0; p < MP; ++p) {
+    const float2 x = a[p][S];
+    const float2 xs = __fmul2_rn(x, make_float2(scale, scale));
+    const int r0 = 8 * p + 2 * c.rg;
+    float2 l = xs;
+    if (p == q0) {
+      l.x = r0 > k ? xs.x : 0.f;
+      l.y = r0 + 1 > k ? xs.y : 0.f;
+    }
+    if (own) {
+      a[p][S] = p == q0 ? make_float2(r0 > k ? xs.x : x.x, r0 + 1 > k ? xs.y : x.y) : xs;
+      *reinterpret_cast<float2 *>(lp + 2 * (p - q0)) = l;
+    }
+  }
+}
+
+// elimination of block B, panel P (columns 4P .. 4P + 3 in slot s), with a
+// one-column look-ahead: step k updates the slot holding column k+1 first
+// and forms that pivot's reciprocal while the other slots are updated.
+// `scale` enters as the reciprocal of column 4P's pivot.
 template <int B, int P>
-__device__ __forceinline__ void panels(Ctx &c, Tile &a) {
+__device__ __forceinline__ void panels(Ctx &c, Tile &a, float scale) {
   constexpr int P0 = blk_c0(B) / 4, NS = blk_ns(B);
   if constexpr (P < P0 + NS) {
-    constexpr int s = P - P0, q0 = P / 2;
+    constexpr int s = P - P0;
 #pragma unroll 1
-    for (int kk = 0; kk < 4; ++kk) {
+    for (int kk = 0; kk < 3; ++kk) {
       const int k = 4 * P + kk;
-      const int kr = 4 * (P % 2) + kk;
-      // the pivot, from the lane holding row k of column group kk
-      const float px = (kr & 1) ? a[q0][s].y : a[q0][s].x;
-      const float piv = __shfl_sync(0xffffffffu, px, (c.lane & 16) | (kk * 4) | (kr >> 1));
-      const bool z = piv == 0.f;
-      const float scale = z ? 0.f : __fdiv_rn(1.0f, piv);
-      c.info = (c.info == 0 && z) ? k + 1 : c.info;
-      // column k: l = a * scale below the pivot (owner column group)
-      const bool own = c.cg == kk;
       float *lp = lptr<P>(c, kk);
-#pragma unroll
-      for (int p = q0; p < MP; ++p) {
-        const float2 x = a[p][s];
-        const float2 xs = __fmul2_rn(x, make_float2(scale, scale));
-        const int r0 = 8 * p + 2 * c.rg;
-        float2 l = xs;
-        if (p == q0) {
-          l.x = r0 > k ? xs.x : 0.f;
-          l.y = r0 + 1 > k ? xs.y : 0.f;
-        }
-        if (own) {
-          a[p][s] = p == q0 ? make_float2(r0 > k ? xs.x : x.x, r0 + 1 > k ? xs.y : x.y) : xs;
-          *reinterpret_cast<float2 *>(lp + 2 * (p - q0)) = l;
-        }
-      }
+      publish_l<P, s>(c, a, kk, scale, lp);
       wsync();
-      lapply<P, s, NS, true>(c, a, lp, kk);
-      // the two-entry ring (columns >= 40) is rewritten two steps later;
-      // the kept columns are never rewritten
-      if constexpr (P >= kKeepP) wsync();
+      lapply<P, s, s + 1, true>(c, a, lp, kk);
+      scale = pivot_scale<P, s>(c, a, kk + 1, k + 1);
+      lapply<P, s + 1, NS, false>(c, a, lp, kk);
+    }
+    {
+      const int k = 4 * P + 3;
+      float *lp = lptr<P>(c, 3);
+      publish_l<P, s>(c, a, 3, scale, lp);
+      wsync();
+      if constexpr (s + 1 < NS) {
+        lapply<P, s + 1, s + 2, false>(c, a, lp, 3);
+        scale = pivot_scale<P + 1, s + 1>(c, a, 0, k + 1);
+        lapply<P, s + 2, NS, false>(c, a, lp, 3);
+      }
     }
     store_slot<B, s>(c, a);
     load_slot<B + 1, s>(c, a);
-    panels<B, P + 1>(c, a);
+    panels<B, P + 1>(c, a, scale);
   }
 }
 
@@ -179,7 +207,8 @@ __device__ __forceinline__ void do_block(Ctx &c, Tile &a) {
   if constexpr (B == 0 || blk_ns(B - 1) <= 2) load_slot<B, 2>(c, a);
   if constexpr (B == 0 || blk_ns(B - 1) <= 3) load_slot<B, 3>(c, a);
   left<B, 0>(c, a);
-  panels<B, blk_c0(B) / 4>(c, a);
+  const float scale = pivot_scale<blk_c0(B) / 4, 0>(c, a, 0, blk_c0(B));
+  panels<B, blk_c0(B) / 4>(c, a, scale);
   wsync();
 }
 
