@@ -245,7 +245,8 @@ def test_lu_kernel_names(lib):
     lib.bqr_lu_kernel_name.argtypes = [ctypes.c_int] * 5
     lib.bqr_lu_kernel_name.restype = ctypes.c_char_p
     assert lib.bqr_lu_kernel_name(0, 56, 56, 0, 0) == b"lll_f32_56x56_left4_x2"
-    assert lib.bqr_lu_kernel_name(0, 56, 56, 1, 1) == b"lu_rf_R8G4_7x15_x2"
+    assert lib.bqr_lu_kernel_name(0, 56, 56, 1, 1) == b"llgj_f32_56x57_left4_x2"
+    assert lib.bqr_lu_kernel_name(0, 56, 56, 2, 1) == b"lu_rf_R8G4_7x15_x2"
     assert lib.bqr_lu_kernel_name(1, 56, 56, 0, 0) == b"lu_rf_R16G8_4x8"
     assert lib.bqr_lu_kernel_name(0, 8, 8, 0, 0) == b"lu_rf_R4G4_2x2_x4"
     assert lib.bqr_lu_kernel_name(0, 129, 129, 0, 0) == b""

@@ -121,3 +121,61 @@ def test_lu56_batches(batch):
     idx = sorted(set(range(0, batch, 53)) | {batch - 1})
     rep = compare_lu(A[idx], 56, out[idx], info[idx])
     assert rep["ok"], rep
+
+
+# ------------------------------------------------------------ left-looking Gauss-Jordan (bqr_llgj.cuh)
+def _gj_gpu(A_cm, B_cm):
+    batch, n, lda = A_cm.shape
+    _, nrhs, ldb = B_cm.shape
+    a = torch.from_numpy(np.ascontiguousarray(A_cm)).cuda()
+    b = torch.from_numpy(np.ascontiguousarray(B_cm)).cuda()
+    info = torch.full((batch,), -7, dtype=torch.int32, device="cuda")
+    st = bqr.load().bqr_gauss_jordan_batched(bqr.R32, n, nrhs, batch, ctypes.c_void_p(a.data_ptr()), lda,
+                                             ctypes.c_void_p(b.data_ptr()), ldb, ctypes.c_void_p(info.data_ptr()),
+                                             None)
+    assert st == 0, st
+    torch.cuda.synchronize()
+    return a.cpu().numpy(), b.cpu().numpy(), info.cpu().numpy()
+
+
+def test_gj56_dispatch():
+    assert bqr.load().bqr_lu_kernel_name(bqr.R32, 56, 56, 1, 1).decode() == "llgj_f32_56x57_left4_x2"
+
+
+@pytest.mark.parametrize("batch", [1, 3, 37, 10067])
+def test_gj56_batches(batch):
+    from oracle.compare import compare_gj
+    A = bqr_inputs.diag_dominant_batch(56, batch, "f32", seed=1200 + batch)
+    B = bqr_inputs.rhs_batch(56, 1, batch, "f32", seed=1300 + batch)
+    Ao, X, info = _gj_gpu(A, B)
+    idx = sorted(set(range(0, batch, 53)) | {batch - 1})
+    rep = compare_gj(A[idx], B[idx], Ao[idx], X[idx], info[idx])
+    assert rep["ok"], rep
+
+
+def test_gj56_zero_pivot_info():
+    """row 30 zero left of and on the diagonal: pivot 30 is exactly zero after
+    the eliminations (scale 0, info 31, the elimination goes on, reading L1);
+    matrix 0 has a zero first pivot (info 1)"""
+    from oracle.compare import compare_gj
+    A = bqr_inputs.diag_dominant_batch(56, 4, "f32", seed=561)
+    B = bqr_inputs.rhs_batch(56, 1, 4, "f32", seed=562)
+    A[1, :31, 30] = 0.0
+    A[0, 0, :] = 0.0
+    Ao, X, info = _gj_gpu(A, B)
+    assert list(info[:2]) == [1, 31] and list(info[2:]) == [0, 0]
+    rep = compare_gj(A, B, Ao, X, info)
+    assert rep["ok"], rep
+
+
+@pytest.mark.parametrize("lda,ldb", [(58, 60), (57, 56), (56, 57)])
+def test_gj56_leading_dims(lda, ldb):
+    """even lda / ldb: the left-looking class; an odd one: lu_rf_kernel"""
+    from oracle.compare import compare_gj
+    A = bqr_inputs.diag_dominant_batch(56, 21, "f32", seed=lda + ldb, lda=lda)
+    B = bqr_inputs.rhs_batch(56, 1, 21, "f32", seed=ldb, ldb=ldb) if "ldb" in bqr_inputs.rhs_batch.__code__.co_varnames \
+        else np.pad(bqr_inputs.rhs_batch(56, 1, 21, "f32", seed=ldb), ((0, 0), (0, 0), (0, ldb - 56)),
+                    constant_values=np.nan)
+    Ao, X, info = _gj_gpu(A, B)
+    rep = compare_gj(A, B, Ao, X, info)
+    assert rep["ok"], rep
