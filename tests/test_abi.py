@@ -250,3 +250,28 @@ def test_lu_kernel_names(lib):
     assert lib.bqr_lu_kernel_name(1, 56, 56, 0, 0) == b"lu_rf_R16G8_4x8"
     assert lib.bqr_lu_kernel_name(0, 8, 8, 0, 0) == b"lu_rf_R4G4_2x2_x4"
     assert lib.bqr_lu_kernel_name(0, 129, 129, 0, 0) == b""
+
+
+def test_left_looking_kernels_sass(lib):
+    """The round-2 left-looking classes (C3 QR, L56 LU, GJ56 Gauss-Jordan):
+    no divergence-guarded shuffles (BRA.DIV / WARPSYNC: their matrix loop
+    runs on a shuffle-broadcast warp index), packed FP32 (FFMA2) in their
+    updates, and at most 96 registers (17 warps = 34 matrices per SM; a
+    scheduler holds 5 warps, 5 x 32 x 96 <= 16384)."""
+    import re
+    import shutil
+    import subprocess
+    exe = shutil.which("cuobjdump") or "/usr/local/cuda/bin/cuobjdump"
+    if not os.path.exists(exe):
+        pytest.skip("cuobjdump not available")
+    names = {"_ZN3bqr2ll17geqrf_ll56_kernelENS0_6LlArgsE": "ll",
+             "_ZN3bqr3lll18getrf_lll56_kernelENS0_4ArgsE": "lll",
+             "_ZN3bqr4llgj16gj_llgj56_kernelENS0_4ArgsE": "llgj"}
+    res = subprocess.run([exe, "-res-usage", bqr._LIB_PATH], capture_output=True, text=True, timeout=600).stdout
+    for mangled in names:
+        sass = subprocess.run([exe, "-sass", "-fun", mangled, bqr._LIB_PATH], capture_output=True, text=True,
+                              timeout=600).stdout
+        assert "FFMA2" in sass, mangled
+        assert "BRA.DIV" not in sass and "WARPSYNC" not in sass, mangled
+        m = re.search(re.escape(mangled) + r".*?\n\s*REG:(\d+)", res, re.S)
+        assert m and int(m.group(1)) <= 96, (mangled, m and m.group(1))
