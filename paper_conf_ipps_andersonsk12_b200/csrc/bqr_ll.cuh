@@ -112,10 +112,6 @@ __device__ __forceinline__ float2 lds64(const float *p) {
   asm volatile("ld.shared.v2.f32 {%0,%1}, [%2];" : "=f"(v.x), "=f"(v.y) : "r"(s));
   return v;
 }
-__device__ __forceinline__ void sts64(float *p, float2 v) {
-  const unsigned s = (unsigned)__cvta_generic_to_shared(p);
-  asm volatile("st.shared.v2.f32 [%0], {%1,%2};" ::"r"(s), "f"(v.x), "f"(v.y) : "memory");
-}
 
 #ifdef BQR_LL_TIMING
 // debug builds only: clock64 stamps of CTA 0's warps (first matrix pair):
@@ -246,10 +242,6 @@ __device__ __forceinline__ void apply(const Ctx &c, Tile &a, const float *vp, fl
       if (MASK0 && j == 0) t = c.cg > kk ? t : 0.f;
       nt[j] = make_float2(-t, -t);
     }
-#endif
-#ifdef BQR_LL_RELOAD
-#pragma unroll
-    for (int p = Q0; p < MP; ++p) v[p] = lds64(vp + 2 * (p - Q0));
 #endif
 #pragma unroll
     for (int p = Q0; p < MP; ++p)
