@@ -155,6 +155,12 @@ using Tile = float2[MP][NSMAX];
 #define BQR_LL_UNROLL_LEFT 4
 #endif
 constexpr int kUnrollLeft = BQR_LL_UNROLL_LEFT;
+// one butterfly for the look-ahead dot and the next column's norm
+// (apply1_look / reflector_fused): parity green but slower on B200 (79.4 vs
+// 69.7 us: 100 B of spills at the 96-register cap, 15% more code), off
+#ifndef BQR_LL_FUSED
+#define BQR_LL_FUSED 0
+#endif
 #ifndef BQR_LL_LOADLAG
 #define BQR_LL_LOADLAG 0
 #endif
@@ -305,6 +311,72 @@ __device__ __forceinline__ void publish(const Ctx &c, Tile &a, const Reflector<f
   if (own && c.rg == 0) *tslot = h.tau;
 }
 
+// ---------------------------------------------------------------- fused look-ahead
+// H_k on the single slot S holding column k+1, returning alongside the dot
+// gamma = sum_{r >= k} a_r^2 of this lane's column BEFORE the update (one
+// butterfly for both): H_k is orthogonal on rows >= k, so after it the
+// squared norm below row k+1 is gamma - a'_k^2 - a'_{k+1}^2 (reflector_fused)
+template <int Q0, int S, bool MASK0>
+__device__ __forceinline__ float apply1_look(const Ctx &c, Tile &a, const float *vp, float tau, int kk, int k) {
+  float2 v[MP];
+#pragma unroll
+  for (int p = Q0; p < MP; ++p) v[p] = lds64(vp + 2 * (p - Q0));
+  float2 w = make_float2(0.f, 0.f), g = make_float2(0.f, 0.f);
+#pragma unroll
+  for (int p = Q0; p < MP; ++p) {
+    w = fma2(v[p], a[p][S], w);
+    float2 x = a[p][S];
+    if (p == Q0) {
+      const int r0 = 8 * p + 2 * c.rg;
+      x.x = r0 >= k ? x.x : 0.f;
+      x.y = r0 + 1 >= k ? x.y : 0.f;
+    }
+    g = fma2(x, x, g);
+  }
+  float sd = w.x + w.y, gg = g.x + g.y;
+  sd += __shfl_xor_sync(0xffffffffu, sd, 1);
+  gg += __shfl_xor_sync(0xffffffffu, gg, 1);
+  sd += __shfl_xor_sync(0xffffffffu, sd, 2);
+  gg += __shfl_xor_sync(0xffffffffu, gg, 2);
+  float t = tau * sd;
+  if (MASK0) t = c.cg > kk ? t : 0.f;
+  const float2 nt = make_float2(-t, -t);
+#pragma unroll
+  for (int p = Q0; p < MP; ++p) a[p][S] = fma2(v[p], nt, a[p][S]);
+  return gg;
+}
+
+// xLARFG of column kn = 4 PP + kkn (slot S) from gamma: sigma = gamma -
+// a'_{kn-1}^2 - alpha^2, accurate while it cancels at most one bit; a
+// warp-uniform fallback to the direct norm (reflector) otherwise, which also
+// keeps tau = 0 exact for an already triangular column (reading Q5)
+template <int PP, int S>
+__device__ __forceinline__ Reflector<float> reflector_fused(const Ctx &c, const Tile &a, int kkn, float gam) {
+  const int kn = 4 * PP + kkn, k = kn - 1;
+  constexpr int qn = PP / 2;
+  // pair of row k: qn, or the previous pair when kn opens an even panel
+  const int krow = k & 7, knrow = kn & 7;
+  float xk_own, xa_own;
+  {
+    const float2 pn = a[qn][S];
+    xa_own = (knrow & 1) ? pn.y : pn.x;
+    if constexpr (PP % 2 == 0 && qn > 0) {
+      const float2 pk = kkn == 0 ? a[qn - 1][S] : pn;
+      xk_own = (krow & 1) ? pk.y : pk.x;
+    } else {
+      xk_own = (krow & 1) ? pn.y : pn.x;
+    }
+  }
+  const float xk = __shfl_sync(0xffffffffu, xk_own, (c.lane & ~3) | (krow >> 1));
+  const float xa = __shfl_sync(0xffffffffu, xa_own, (c.lane & ~3) | (knrow >> 1));
+  const float nu2 = fmaf(-xk, xk, gam);
+  const float sig = fmaf(-xa, xa, nu2);
+  const bool own = c.cg == kkn;
+  const bool bad = own && !(nu2 >= 0.5f * gam && sig >= 0.0625f * nu2);
+  if (__any_sync(0xffffffffu, bad)) return reflector<PP, S>(c, a, kkn);
+  return make_reflector(xa, sig);
+}
+
 // ---------------------------------------------------------------- phases
 // left-looking: H_0 .. H_{c0-1} (panels 0 .. c0/4 - 1) on block B
 // H_{k+1} H_k on slots [0, NS) in one pass (k even, both of panel P, rows
@@ -408,8 +480,13 @@ __device__ __forceinline__ void panels(const Ctx &c, Tile &a) {
       const int k = 4 * P + kk;
       const float tau = taus[k];
       const float *vp = vptr<P>(c, kk);
+#if BQR_LL_FUSED
+      const float gam = apply1_look<q0, s, true>(c, a, vp, tau, kk, k);
+      const Reflector<float> h = reflector_fused<P, s>(c, a, kk + 1, gam);
+#else
       apply<q0, s, s + 1, true>(c, a, vp, tau, kk);
       const Reflector<float> h = reflector<P, s>(c, a, kk + 1);
+#endif
       apply<q0, s + 1, NS, false>(c, a, vp, tau, kk);
       publish<P, s>(c, a, h, kk + 1, vptr<P>(c, kk + 1), taus + k + 1);
     }
@@ -430,8 +507,13 @@ __device__ __forceinline__ void panels(const Ctx &c, Tile &a) {
       const int k = 4 * P + 3;
       const float tau = taus[k];
       const float *vp = vptr<P>(c, 3);
+#if BQR_LL_FUSED
+      const float gam = apply1_look<q0, s + 1, false>(c, a, vp, tau, 3, k);
+      const Reflector<float> h = reflector_fused<P + 1, s + 1>(c, a, 0, gam);
+#else
       apply<q0, s + 1, s + 2, false>(c, a, vp, tau, 3);
       const Reflector<float> h = reflector<P + 1, s + 1>(c, a, 0);
+#endif
       apply<q0, s + 2, NS, false>(c, a, vp, tau, 3);
       publish<P + 1, s + 1>(c, a, h, 0, vptr<P + 1>(c, 0), taus + k + 1);
     }
