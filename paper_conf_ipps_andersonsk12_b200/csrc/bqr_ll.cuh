@@ -151,8 +151,12 @@ __device__ __forceinline__ float *vptr(const Ctx &c, int kk) {
 
 using Tile = float2[MP][NSMAX];
 
+// unroll of the left-looking reflector loop.  1 keeps the kernel at 5.3k
+// SASS instructions (9.2k at 4): the same full-batch time (69.8 us), but a
+// cold instruction cache after the L2 flush costs a lone warp 25 us less
+// (batch 1: 30.8 vs 62.4 us; batch 625: 32.8 vs 54.3 us)
 #ifndef BQR_LL_UNROLL_LEFT
-#define BQR_LL_UNROLL_LEFT 4
+#define BQR_LL_UNROLL_LEFT 1
 #endif
 constexpr int kUnrollLeft = BQR_LL_UNROLL_LEFT;
 // one butterfly for the look-ahead dot and the next column's norm
