@@ -61,7 +61,7 @@ using namespace bqr::host;
 // classes, then fp32, then complex64, then the
 // experiment-only alternatives (BQR_FORCE_VARIANT).
 struct Tables {
-  static constexpr int kN = 7;
+  static constexpr int kN = 8;
   const ClassEntry *t[kN];
   int n[kN];
   Tables() {
@@ -72,6 +72,7 @@ struct Tables {
     t[4] = classes_f32(&n[4]);
     t[5] = classes_c64(&n[5]);
     t[6] = classes_alt(&n[6]);
+    t[7] = classes_cl(&n[7]);
   }
   template <class F>
   const Plan *find(F pred) const {

@@ -202,6 +202,7 @@ int apply_dispatch(const ApplyArgs &a, cudaStream_t s) {
 // class tables (one translation unit each) and the tiny / apply entry points
 const ClassEntry *classes_ll(int *n);
 const ClassEntry *classes_llc(int *n);
+const ClassEntry *classes_cl(int *n);
 const ClassEntry *classes_co(int *n);
 const ClassEntry *classes_headline(int *n);
 const ClassEntry *classes_f32(int *n);
