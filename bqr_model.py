@@ -195,8 +195,9 @@ def bounds_us(L: Layout, batch: int, instr_total: float, cpi_warp: float, useful
     hi = ceil(rounds) x (the chain fully exposed + the instructions of one
          warp per round x the measured warp CPI, ncu "warp cycles per issued
          instruction", i.e. the issue stalls of this kernel at its
-         occupancy): every round paid at full contention, the last (partial)
-         one included, nothing of the chain hidden.
+         occupancy, x the busiest scheduler's share of the SM's warps over
+         the mean share): every round paid at full contention, the last
+         (partial) one included, nothing of the chain hidden.
     The per-matrix latency floor (batch 1, the strong-scaling limit) is the
     chain plus one warp's instructions at CPI 1 (lo1) ... at the measured
     CPI (hi1).  The hi bounds add the measured launch / event overhead of an
@@ -211,12 +212,21 @@ def bounds_us(L: Layout, batch: int, instr_total: float, cpi_warp: float, useful
     issue = instr_total / (lat["schedulers"] * n_sm)
     fma = useful_fmas / (lat["fma_per_clk_sm"] * n_sm)
     lo = max(issue, fma, math.ceil(rounds - 1e-9) * chain)
-    hi = math.ceil(rounds - 1e-9) * (chain + per_warp_round * cpi_warp)
+    # the measured CPI is the mean over all warps; a scheduler holding
+    # ceil(w/4) of an SM's w warps (17 warps: 5 on one, 4.25 on average)
+    # stretches its warps' stalls by that ratio, and the launch lasts as long
+    # as its slowest warp (profiles/r02/ll/timeline_full_batch.txt: the
+    # 5-warp scheduler's warps finish ~10% after the others)
+    wps = max(1.0, min(float(L.resident), batch / n_sm) * L.warps_per_matrix)
+    per_sched = wps / lat["schedulers"]
+    skew = max(1.0, math.ceil(per_sched - 1e-9) / per_sched) if per_sched >= 1.0 else 1.0
+    hi = math.ceil(rounds - 1e-9) * (chain + per_warp_round * cpi_warp * skew)
     # an event-timed launch also carries the launch / event overhead (an
     # empty kernel measures 4.96 us min between two CUDA events on B200)
     return {"rounds": rounds, "lo_us": lo / f, "hi_us": hi / f + lat["launch_event_us"],
             "lo_terms_us": {"issue": issue / f, "fp32_pipe": fma / f, "chain": math.ceil(rounds - 1e-9) * chain / f},
             "chain_cycles_per_matrix": chain, "instr_per_warp_round": per_warp_round, "cpi_warp": cpi_warp,
+            "scheduler_skew": skew,
             "latency_floor_us": {"lo": (chain + per_warp_round) / f,
                                  "hi": (chain + per_warp_round * cpi_warp) / f + lat["launch_event_us"]}}
 
