@@ -27,6 +27,16 @@
 #include <cooperative_groups.h>
 #include "bqr_common.cuh"
 
+// LAZY: the owner of column k+2 applies v_k to that column only and defers
+// the rest of step k until after its look-ahead at step k+1.  Parity green
+// but slower on B200 (cl1 86 vs 72 us, cl4 72 vs 60 us at batch 32): the
+// owner of k+2 already finishes its remainder while the owner of k+1 runs
+// the look-ahead chain, so deferring only moves work (profiles/r02/
+// experiments/c4_cluster.jsonl)
+#ifndef BQR_CL_LAZY
+#define BQR_CL_LAZY 0
+#endif
+
 namespace bqr {
 namespace cl {
 
@@ -162,37 +172,11 @@ struct Kernel {
     for (int i = 0; i < MR; ++i) a[i][S] = X::fnms(v[i], tw, a[i][S]);
   }
 
-  // step k (pivot slot S0 of its owner): wait for v_k, look-ahead on column
-  // k+1 (its owner), then every other live column of this warp
+  // H_kk^H on every live slot of this warp (column > kk, < ncol, != excl),
+  // slots below S0 hold no such column
   template <int S0>
-  static __device__ __forceinline__ void step(Ctx &c, Tile &a, int k, int ncol) {
-    const int g = c.gbase + k;
-    const int b = g % NBUF;
-    while (!cl_try_wait(c.full + b, (unsigned)(g / NBUF) & 1u)) {
-    }
-    float2 v[MR];
-#pragma unroll
-    for (int i = 0; i < MR; ++i) v[i] = c.vbuf[b * C::MMAX + c.lane + 32 * i];
-    const float2 ct = X::conj(c.tbuf[b]);
-    // the local arrival of ring entry g + NBUF - 1 (its previous phase, g - 1,
-    // has completed: this warp waited for it)
-    if (threadIdx.x == 0 && k + NBUF - 1 < c.p->kmax) cl_expect(c.full + (g + NBUF - 1) % NBUF, C::kStepBytes);
-    const int k1 = k + 1;
-    const bool look = k1 < c.p->kmax && c.gcg == k1 % G;
-    // the look-ahead column's slot: S0 (same sweep) or S0 + 1 (next sweep)
-    const bool nextsweep = (k1 % G) == 0;
-    if (look) {
-      if (nextsweep) {
-        if constexpr (S0 + 1 < NC) {
-          apply1<S0 + 1>(a, v, ct);
-          reflect_publish<S0 + 1>(c, a, k1);
-        }
-      } else {
-        apply1<S0>(a, v, ct);
-        reflect_publish<S0>(c, a, k1);
-      }
-    }
-    // remaining live slots: column gcg + G s > k, < ncol, not the look-ahead one
+  static __device__ __forceinline__ void rest(Ctx &c, Tile &a, const float2 (&v)[MR], float2 ct, int kk, int excl,
+                                              int ncol) {
     float wv[2 * NC];
 #pragma unroll
     for (int s = 0; s < NC; ++s) {
@@ -209,9 +193,7 @@ struct Kernel {
     for (int s = 0; s < NC; ++s) {
       if (s < S0) continue;
       const int col = c.gcg + G * s;
-      const bool lookslot = look && (nextsweep ? s == S0 + 1 : s == S0);
-      const bool live = col > k && col < ncol && !lookslot;
-      if (live) {
+      if (col > kk && col < ncol && col != excl) {
         const float2 tw = X::mul(ct, make_float2(wv[2 * s], wv[2 * s + 1]));
 #pragma unroll
         for (int i = 0; i < MR; ++i) a[i][s] = X::fnms(v[i], tw, a[i][s]);
@@ -219,16 +201,74 @@ struct Kernel {
     }
   }
 
+  // H_k^H on column kc only (its slot is S0 or S0 + 1)
   template <int S0>
-  static __device__ __forceinline__ void sweep(Ctx &c, Tile &a, int ncol) {
+  static __device__ __forceinline__ void apply_col(Tile &a, const float2 (&v)[MR], float2 ct, int kc) {
+    if (kc / G != S0) {
+      if constexpr (S0 + 1 < NC) apply1<S0 + 1>(a, v, ct);
+    } else {
+      apply1<S0>(a, v, ct);
+    }
+  }
+
+  // step k (pivot slot S0 of its owner): wait for v_k; the owner of column
+  // k+1 updates it and publishes reflector k+1 (look-ahead), then every
+  // warp applies v_k to its other columns (with BQR_CL_LAZY, the owner of
+  // column k+2 defers that remainder past its own look-ahead at step k+1).
+  template <int S0>
+  static __device__ __forceinline__ void step(Ctx &c, Tile &a, int k, int ncol, float2 (&vd)[MR], float2 &ctd,
+                                              bool &defer) {
+    const int g = c.gbase + k;
+    const int b = g % NBUF;
+    while (!cl_try_wait(c.full + b, (unsigned)(g / NBUF) & 1u)) {
+    }
+    float2 v[MR];
+#pragma unroll
+    for (int i = 0; i < MR; ++i) v[i] = c.vbuf[b * C::MMAX + c.lane + 32 * i];
+    const float2 ct = X::conj(c.tbuf[b]);
+    // the local arrival of ring entry g + NBUF - 1 (its previous phase, g - 1,
+    // has completed: this warp waited for it)
+    if (threadIdx.x == 0 && k + NBUF - 1 < c.p->kmax) cl_expect(c.full + (g + NBUF - 1) % NBUF, C::kStepBytes);
+    const int k1 = k + 1, k2 = k + 2;
+    const bool look = k1 < c.p->kmax && c.gcg == k1 % G;
+    if (look) {
+      if (k1 / G != S0) {
+        if constexpr (S0 + 1 < NC) {
+          apply1<S0 + 1>(a, v, ct);
+          reflect_publish<S0 + 1>(c, a, k1);
+        }
+      } else {
+        apply1<S0>(a, v, ct);
+        reflect_publish<S0>(c, a, k1);
+      }
+    }
+#if BQR_CL_LAZY
+    if (!look && k2 < c.p->kmax && c.gcg == k2 % G) {
+      apply_col<S0>(a, v, ct, k2);
+#pragma unroll
+      for (int i = 0; i < MR; ++i) vd[i] = v[i];
+      ctd = ct;
+      defer = true;
+      return;
+    }
+    if (defer) {
+      rest<S0>(c, a, vd, ctd, k - 1, k1, ncol);
+      defer = false;
+    }
+#endif
+    rest<S0>(c, a, v, ct, k, look ? k1 : -1, ncol);
+  }
+
+  template <int S0>
+  static __device__ __forceinline__ void sweep(Ctx &c, Tile &a, int ncol, float2 (&vd)[MR], float2 &ctd, bool &defer) {
     if constexpr (S0 < NC) {
 #pragma unroll 1
       for (int r0 = 0; r0 < G; ++r0) {
         const int k = S0 * G + r0;
         if (k >= c.p->kmax) return;
-        step<S0>(c, a, k, ncol);
+        step<S0>(c, a, k, ncol, vd, ctd, defer);
       }
-      sweep<S0 + 1>(c, a, ncol);
+      sweep<S0 + 1>(c, a, ncol, vd, ctd, defer);
     }
   }
 
@@ -276,7 +316,12 @@ struct Kernel {
       if (threadIdx.x == 0)
         for (int j = 0; j < NBUF - 1 && j < p.kmax; ++j) cl_expect(c.full + (c.gbase + j) % NBUF, C::kStepBytes);
       if (c.gcg == 0 && p.kmax > 0) reflect_publish<0>(c, a, 0);
-      sweep<0>(c, a, ncol);
+      float2 vd[MR];
+      float2 ctd = X::zero();
+      bool defer = false;
+#pragma unroll
+      for (int i = 0; i < MR; ++i) vd[i] = X::zero();
+      sweep<0>(c, a, ncol, vd, ctd, defer);
 #pragma unroll
       for (int s = 0; s < NC; ++s) {
         const int col = c.gcg + G * s;

@@ -5,6 +5,7 @@ STAP shape 240 x 66 c64.  Each variant runs in its own process
 (BQR_FORCE_VARIANT is read once per process).
 
     python tools/cl_probe.py [default alt_cl4_c64_256x72_aug alt_cl2_c64_256x72_aug]
+    CL_PROBE_LIB=abl/libbqr_X.so python tools/cl_probe.py ...   (an experiment build)
 """
 import os
 import subprocess
@@ -16,13 +17,16 @@ for var in variants:
     code = f"""
 import sys, json, ctypes; sys.path.insert(0, {ROOT!r}); sys.path.insert(0, {os.path.join(ROOT, 'tests')!r})
 import torch, numpy as np
+import os
 import paper_conf_ipps_andersonsk12_b200 as bqr
+if os.environ.get('CL_PROBE_LIB'):
+    bqr._LIB_PATH = os.path.abspath(os.environ['CL_PROBE_LIB'])
 import bqr_inputs
 from oracle.compare import compare_geqrf, compare_apply
 from gpu_util import geqrf_gpu, geqrf_qhb_gpu
 var = {var!r}
 lib = bqr.load()
-row = {{'variant': var, 'kernel': bqr.kernel_name(bqr.C64, 240, 66),
+row = {{'variant': var, 'lib': os.environ.get('CL_PROBE_LIB', 'in-tree'), 'kernel': bqr.kernel_name(bqr.C64, 240, 66),
        'qhb_kernel': lib.bqr_qhb_kernel_name(bqr.C64, 240, 66, 1).decode()}}
 par = []
 for (m, n, b, seed) in ((240, 66, 5, 1), (240, 66, 37, 2), (256, 72, 3, 3), (200, 50, 4, 4), (97, 13, 3, 5)):
@@ -48,7 +52,8 @@ for b in (1, 16, 32, 37, 64, 74, 148, 256):
     ts = []
     for it in range(13):
         A.copy_(A0)
-        big.zero_()
+        if not os.environ.get('CL_PROBE_NOFLUSH'):
+            big.zero_()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(s)
         st = bqr.geqrf_batched_ptr(bqr.C64, 240, 66, b, A.data_ptr(), 240, tau.data_ptr(), s.cuda_stream)
@@ -58,7 +63,7 @@ for b in (1, 16, 32, 37, 64, 74, 148, 256):
         if it >= 3:
             ts.append(e0.elapsed_time(e1) * 1e3)
     times[b] = round(sorted(ts)[len(ts) // 2], 2)
-row['geqrf_us_flushed'] = times
+row['geqrf_us_noflush' if os.environ.get('CL_PROBE_NOFLUSH') else 'geqrf_us_flushed'] = times
 print(json.dumps(row), flush=True)
 """
     env = dict(os.environ)
