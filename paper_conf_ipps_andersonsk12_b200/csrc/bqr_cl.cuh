@@ -36,6 +36,12 @@
 #ifndef BQR_CL_LAZY
 #define BQR_CL_LAZY 0
 #endif
+// FUSED: look_fused (one butterfly for the look-ahead dot and the next
+// column's norm).  Parity green but slower on B200 (cl4 71.7 vs 61.4 us,
+// cl1 73.7 vs 71.7 us at batch 32): off
+#ifndef BQR_CL_FUSED
+#define BQR_CL_FUSED 0
+#endif
 
 namespace bqr {
 namespace cl {
@@ -138,6 +144,13 @@ struct Kernel {
     }
 #pragma unroll
     for (int o = 16; o >= 1; o >>= 1) sg += __shfl_xor_sync(0xffffffffu, sg, o);
+    publish<S>(c, a, k, alpha, sg);
+  }
+
+  // xLARFG from alpha and sigma = sum_{r>k} |a_rk|^2, column k (slot S)
+  // scaled in place, v and tau published
+  template <int S>
+  static __device__ __forceinline__ void publish(Ctx &c, Tile &a, int k, float2 alpha, float sg) {
     const Reflector<float2> h = make_reflector(alpha, sg);
     float2 v[MR];
 #pragma unroll
@@ -158,6 +171,58 @@ struct Kernel {
       if (c.lane == 0) cl_st_async(cl_mapa(ta, (unsigned)q), h.tau, rb);
     }
     if (c.lane == 0) c.p->tau[c.mat * c.p->strideT + k] = h.tau;
+  }
+
+  // look-ahead on column k1 (slot S) fused with its norm: one butterfly of
+  // w = v^H a together with the pre-update sums over rows r > k1 of |a|^2,
+  // conj(v) a and |v|^2, from which sigma' = sum |a - v t|^2 (t = conj(tau) w)
+  // = saa - 2 Re(conj(t) sva) + |t|^2 svv.  Heavy cancellation
+  // (sigma' < saa / 4) falls back to the direct sum after the update.
+  template <int S>
+  static __device__ __forceinline__ void look_fused(Ctx &c, Tile &a, const float2 (&v)[MR], float2 ct, int k1) {
+    const int kl = k1 & 31, ki = k1 >> 5;
+    float r6[6] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f};  // w.x w.y saa sva.x sva.y svv
+    float2 xa = a[0][S], xv = v[0];
+#pragma unroll
+    for (int i = 0; i < MR; ++i) {
+      const int r = c.lane + 32 * i;
+      const float2 x = a[i][S], y = v[i];
+      const float2 w = X::cfma(y, x, make_float2(r6[0], r6[1]));
+      r6[0] = w.x;
+      r6[1] = w.y;
+      if (i > 0 && i == ki) {
+        xa = x;
+        xv = y;
+      }
+      if (r > k1) {
+        r6[2] = X::abs2_acc(x, r6[2]);
+        const float2 q = X::cfma(y, x, make_float2(r6[3], r6[4]));
+        r6[3] = q.x;
+        r6[4] = q.y;
+        r6[5] = X::abs2_acc(y, r6[5]);
+      }
+    }
+    const float2 alpha0 = X::shfl(xa, kl), v0 = X::shfl(xv, kl);
+    row_allreduce_multi<32, 6>(r6, c.lane);
+    const float2 tw = X::mul(ct, make_float2(r6[0], r6[1]));
+#pragma unroll
+    for (int i = 0; i < MR; ++i) a[i][S] = X::fnms(v[i], tw, a[i][S]);
+    const float2 alpha = X::fnms(v0, tw, alpha0);
+    // Re(conj(t) sva) = t.x sva.x + t.y sva.y
+    const float cross = fmaf(tw.x, r6[3], tw.y * r6[4]);
+    const float t2 = fmaf(tw.x, tw.x, tw.y * tw.y);
+    float sg = fmaf(t2, r6[5], fmaf(-2.f, cross, r6[2]));
+    if (!(sg >= 0.25f * r6[2])) {
+      sg = 0.f;
+#pragma unroll
+      for (int i = 0; i < MR; ++i) {
+        const int r = c.lane + 32 * i;
+        sg = r > k1 ? X::abs2_acc(a[i][S], sg) : sg;
+      }
+#pragma unroll
+      for (int o = 16; o >= 1; o >>= 1) sg += __shfl_xor_sync(0xffffffffu, sg, o);
+    }
+    publish<S>(c, a, k1, alpha, sg);
   }
 
   // a -= v conj(tau) (v^H a) on slot S
@@ -234,12 +299,20 @@ struct Kernel {
     if (look) {
       if (k1 / G != S0) {
         if constexpr (S0 + 1 < NC) {
+#if BQR_CL_FUSED
+          look_fused<S0 + 1>(c, a, v, ct, k1);
+#else
           apply1<S0 + 1>(a, v, ct);
           reflect_publish<S0 + 1>(c, a, k1);
+#endif
         }
       } else {
+#if BQR_CL_FUSED
+        look_fused<S0>(c, a, v, ct, k1);
+#else
         apply1<S0>(a, v, ct);
         reflect_publish<S0>(c, a, k1);
+#endif
       }
     }
 #if BQR_CL_LAZY
