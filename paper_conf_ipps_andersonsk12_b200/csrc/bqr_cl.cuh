@@ -69,6 +69,24 @@ struct Cfg {
   static constexpr unsigned kStepBytes = MMAX * 8 + 8;  // v and tau, per CTA and step
 };
 
+#ifdef BQR_CL_TIMING
+// per-step stamps of the look-ahead owner in the first cluster, first matrix
+// (clock64 of its SM; with CL = 1 every warp is on one SM): [k][0] v_k
+// arrived, [1] dot + update of column k+1 done, [2] norm reduced, [3]
+// reflector k+1 published (stores issued)
+constexpr int kClDbgSteps = 80;
+static __device__ long long g_cl_dbg[kClDbgSteps * 4];
+#define CL_STAMP(c, k, e)                                                                  \
+  do {                                                                                      \
+    if (blockIdx.x < gridDim.x && (c).mat == 0 && (c).lane == 0 && (k) < kClDbgSteps)     \
+      g_cl_dbg[(k) * 4 + (e)] = clock64();                                                  \
+  } while (0)
+#else
+#define CL_STAMP(c, k, e) \
+  do {                    \
+  } while (0)
+#endif
+
 __device__ __forceinline__ unsigned cl_smem_u32(const void *p) { return (unsigned)__cvta_generic_to_shared(p); }
 
 __device__ __forceinline__ unsigned cl_mapa(unsigned a, unsigned rank) {
@@ -144,7 +162,9 @@ struct Kernel {
     }
 #pragma unroll
     for (int o = 16; o >= 1; o >>= 1) sg += __shfl_xor_sync(0xffffffffu, sg, o);
+    CL_STAMP(c, k - 1 < 0 ? 0 : k - 1, 2);
     publish<S>(c, a, k, alpha, sg);
+    CL_STAMP(c, k - 1 < 0 ? 0 : k - 1, 3);
   }
 
   // xLARFG from alpha and sigma = sum_{r>k} |a_rk|^2, column k (slot S)
@@ -235,6 +255,9 @@ struct Kernel {
     const float2 tw = X::mul(ct, w);
 #pragma unroll
     for (int i = 0; i < MR; ++i) a[i][S] = X::fnms(v[i], tw, a[i][S]);
+#ifdef BQR_CL_TIMING
+    if (threadIdx.x % 32 == 0) asm volatile("" ::"f"(a[0][S].x), "f"(a[MR - 1][S].y));
+#endif
   }
 
   // H_kk^H on every live slot of this warp (column > kk, < ncol, != excl),
@@ -297,12 +320,14 @@ struct Kernel {
     const int k1 = k + 1, k2 = k + 2;
     const bool look = k1 < c.p->kmax && c.gcg == k1 % G;
     if (look) {
+      CL_STAMP(c, k, 0);
       if (k1 / G != S0) {
         if constexpr (S0 + 1 < NC) {
 #if BQR_CL_FUSED
           look_fused<S0 + 1>(c, a, v, ct, k1);
 #else
           apply1<S0 + 1>(a, v, ct);
+          CL_STAMP(c, k, 1);
           reflect_publish<S0 + 1>(c, a, k1);
 #endif
         }
@@ -311,6 +336,7 @@ struct Kernel {
         look_fused<S0>(c, a, v, ct, k1);
 #else
         apply1<S0>(a, v, ct);
+        CL_STAMP(c, k, 1);
         reflect_publish<S0>(c, a, k1);
 #endif
       }
