@@ -39,6 +39,12 @@
 // FUSED: look_fused (one butterfly for the look-ahead dot and the next
 // column's norm).  Parity green but slower on B200 (cl4 71.7 vs 61.4 us,
 // cl1 73.7 vs 71.7 us at batch 32): off
+#ifndef BQR_CL_FFMA2
+#define BQR_CL_FFMA2 1
+#endif
+#ifndef BQR_CL_LOCAL
+#define BQR_CL_LOCAL 1
+#endif
 #ifndef BQR_CL_FUSED
 #define BQR_CL_FUSED 0
 #endif
@@ -132,6 +138,9 @@ struct Kernel {
   using C = Cfg<CL, W, NC>;
   using X = El<float2>;
   static constexpr int MR = C::MR, G = C::G, NBUF = C::NBUF;
+  // a one-CTA "cluster" publishes with shared stores + a release.cta arrive
+  // per lane (count 32) instead of st.async + expect_tx
+  static constexpr bool kLocal = CL == 1 && BQR_CL_LOCAL;
   using Tile = float2[MR][NC];
 
   struct Ctx {
@@ -181,14 +190,23 @@ struct Kernel {
       a[i][S] = r > k ? xs : (r == k ? make_float2(h.beta, 0.f) : a[i][S]);
     }
     const int b = (c.gbase + k) % NBUF;
-    const unsigned va = cl_smem_u32(c.vbuf + b * C::MMAX + c.lane), ta = cl_smem_u32(c.tbuf + b),
-                   ba = cl_smem_u32(c.full + b);
+    if constexpr (kLocal) {
+      // one CTA: plain shared stores, each lane's arrive (release.cta) covers them
 #pragma unroll
-    for (int q = 0; q < CL; ++q) {
-      const unsigned rv = cl_mapa(va, (unsigned)q), rb = cl_mapa(ba, (unsigned)q);
+      for (int i = 0; i < MR; ++i) c.vbuf[b * C::MMAX + c.lane + 32 * i] = v[i];
+      if (c.lane == 0) c.tbuf[b] = h.tau;
+      __syncwarp();
+      asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(cl_smem_u32(c.full + b)) : "memory");
+    } else {
+      const unsigned va = cl_smem_u32(c.vbuf + b * C::MMAX + c.lane), ta = cl_smem_u32(c.tbuf + b),
+                     ba = cl_smem_u32(c.full + b);
 #pragma unroll
-      for (int i = 0; i < MR; ++i) cl_st_async(rv + 256u * i, v[i], rb);
-      if (c.lane == 0) cl_st_async(cl_mapa(ta, (unsigned)q), h.tau, rb);
+      for (int q = 0; q < CL; ++q) {
+        const unsigned rv = cl_mapa(va, (unsigned)q), rb = cl_mapa(ba, (unsigned)q);
+#pragma unroll
+        for (int i = 0; i < MR; ++i) cl_st_async(rv + 256u * i, v[i], rb);
+        if (c.lane == 0) cl_st_async(cl_mapa(ta, (unsigned)q), h.tau, rb);
+      }
     }
     if (c.lane == 0) c.p->tau[c.mat * c.p->strideT + k] = h.tau;
   }
@@ -245,16 +263,78 @@ struct Kernel {
     publish<S>(c, a, k1, alpha, sg);
   }
 
-  // a -= v conj(tau) (v^H a) on slot S
+  // packed complex arithmetic (FFMA2 on the (re, im) pair with a broadcast
+  // scalar): conj(v) a summed as P = sum vr (ar, ai), Q = sum vi (ar, ai),
+  // w = (P.x + Q.y, P.y - Q.x); a - v t = a + vr (-tr, -ti) + vi (ti, -tr)
   template <int S>
-  static __device__ __forceinline__ void apply1(Tile &a, const float2 (&v)[MR], float2 ct) {
+  static __device__ __forceinline__ float2 dotS(const float2 (&v)[MR], const Tile &a) {
+#if BQR_CL_FFMA2
+    float2 P = X::zero(), Q = X::zero();
+#pragma unroll
+    for (int i = 0; i < MR; ++i) {
+      P = __ffma2_rn(make_float2(v[i].x, v[i].x), a[i][S], P);
+      Q = __ffma2_rn(make_float2(v[i].y, v[i].y), a[i][S], Q);
+    }
+    return make_float2(P.x + Q.y, P.y - Q.x);
+#else
     float2 w = X::zero();
 #pragma unroll
     for (int i = 0; i < MR; ++i) w = X::cfma(v[i], a[i][S], w);
-    w = cl_allreduce(w);
-    const float2 tw = X::mul(ct, w);
+    return w;
+#endif
+  }
+  template <int S>
+  static __device__ __forceinline__ void updS(const float2 (&v)[MR], float2 tw, Tile &a) {
+#if BQR_CL_FFMA2
+    const float2 n1 = make_float2(-tw.x, -tw.y), n2 = make_float2(tw.y, -tw.x);
+#pragma unroll
+    for (int i = 0; i < MR; ++i) {
+      a[i][S] = __ffma2_rn(make_float2(v[i].x, v[i].x), n1, a[i][S]);
+      a[i][S] = __ffma2_rn(make_float2(v[i].y, v[i].y), n2, a[i][S]);
+    }
+#else
 #pragma unroll
     for (int i = 0; i < MR; ++i) a[i][S] = X::fnms(v[i], tw, a[i][S]);
+#endif
+  }
+
+  static __device__ __forceinline__ float2 dot_slot(const float2 (&v)[MR], const Tile &a, int s) {
+#if BQR_CL_FFMA2
+    float2 P = X::zero(), Q = X::zero();
+#pragma unroll
+    for (int i = 0; i < MR; ++i) {
+      P = __ffma2_rn(make_float2(v[i].x, v[i].x), a[i][s], P);
+      Q = __ffma2_rn(make_float2(v[i].y, v[i].y), a[i][s], Q);
+    }
+    return make_float2(P.x + Q.y, P.y - Q.x);
+#else
+    float2 w = X::zero();
+#pragma unroll
+    for (int i = 0; i < MR; ++i) w = X::cfma(v[i], a[i][s], w);
+    return w;
+#endif
+  }
+  static __device__ __forceinline__ void upd_slot(const float2 (&v)[MR], float2 tw, Tile &a, int s) {
+#if BQR_CL_FFMA2
+    const float2 n1 = make_float2(-tw.x, -tw.y), n2 = make_float2(tw.y, -tw.x);
+#pragma unroll
+    for (int i = 0; i < MR; ++i) {
+      a[i][s] = __ffma2_rn(make_float2(v[i].x, v[i].x), n1, a[i][s]);
+      a[i][s] = __ffma2_rn(make_float2(v[i].y, v[i].y), n2, a[i][s]);
+    }
+#else
+#pragma unroll
+    for (int i = 0; i < MR; ++i) a[i][s] = X::fnms(v[i], tw, a[i][s]);
+#endif
+  }
+
+  // a -= v conj(tau) (v^H a) on slot S
+  template <int S>
+  static __device__ __forceinline__ void apply1(Tile &a, const float2 (&v)[MR], float2 ct) {
+    float2 w = dotS<S>(v, a);
+    w = cl_allreduce(w);
+    const float2 tw = X::mul(ct, w);
+    updS<S>(v, tw, a);
 #ifdef BQR_CL_TIMING
     if (threadIdx.x % 32 == 0) asm volatile("" ::"f"(a[0][S].x), "f"(a[MR - 1][S].y));
 #endif
@@ -269,10 +349,7 @@ struct Kernel {
 #pragma unroll
     for (int s = 0; s < NC; ++s) {
       float2 w = X::zero();
-      if (s >= S0) {
-#pragma unroll
-        for (int i = 0; i < MR; ++i) w = X::cfma(v[i], a[i][s], w);
-      }
+      if (s >= S0) w = dot_slot(v, a, s);
       wv[2 * s] = w.x;
       wv[2 * s + 1] = w.y;
     }
@@ -283,8 +360,7 @@ struct Kernel {
       const int col = c.gcg + G * s;
       if (col > kk && col < ncol && col != excl) {
         const float2 tw = X::mul(ct, make_float2(wv[2 * s], wv[2 * s + 1]));
-#pragma unroll
-        for (int i = 0; i < MR; ++i) a[i][s] = X::fnms(v[i], tw, a[i][s]);
+        upd_slot(v, tw, a, s);
       }
     }
   }
@@ -316,7 +392,7 @@ struct Kernel {
     const float2 ct = X::conj(c.tbuf[b]);
     // the local arrival of ring entry g + NBUF - 1 (its previous phase, g - 1,
     // has completed: this warp waited for it)
-    if (threadIdx.x == 0 && k + NBUF - 1 < c.p->kmax) cl_expect(c.full + (g + NBUF - 1) % NBUF, C::kStepBytes);
+    if (!kLocal && threadIdx.x == 0 && k + NBUF - 1 < c.p->kmax) cl_expect(c.full + (g + NBUF - 1) % NBUF, C::kStepBytes);
     const int k1 = k + 1, k2 = k + 2;
     const bool look = k1 < c.p->kmax && c.gcg == k1 % G;
     if (look) {
@@ -386,7 +462,7 @@ struct Kernel {
     c.p = &p;
     c.gbase = 0;
     if (threadIdx.x < NBUF) {
-      asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(cl_smem_u32(c.full + threadIdx.x)), "r"(1)
+      asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(cl_smem_u32(c.full + threadIdx.x)), "r"(kLocal ? 32 : 1)
                    : "memory");
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
@@ -412,7 +488,7 @@ struct Kernel {
           a[i][s] = x;
         }
       }
-      if (threadIdx.x == 0)
+      if (!kLocal && threadIdx.x == 0)
         for (int j = 0; j < NBUF - 1 && j < p.kmax; ++j) cl_expect(c.full + (c.gbase + j) % NBUF, C::kStepBytes);
       if (c.gcg == 0 && p.kmax > 0) reflect_publish<0>(c, a, 0);
       float2 vd[MR];
