@@ -345,21 +345,22 @@ struct Kernel {
   template <int S0>
   static __device__ __forceinline__ void rest(Ctx &c, Tile &a, const float2 (&v)[MR], float2 ct, int kk, int excl,
                                               int ncol) {
-    float wv[2 * NC];
+    // only slots S0 .. NC-1 can hold live columns: reduce just those
+    constexpr int NL = NC - S0;
+    float wv[2 * NL];
 #pragma unroll
-    for (int s = 0; s < NC; ++s) {
-      float2 w = X::zero();
-      if (s >= S0) w = dot_slot(v, a, s);
-      wv[2 * s] = w.x;
-      wv[2 * s + 1] = w.y;
+    for (int j = 0; j < NL; ++j) {
+      const float2 w = dot_slot(v, a, S0 + j);
+      wv[2 * j] = w.x;
+      wv[2 * j + 1] = w.y;
     }
-    row_allreduce_multi<32, 2 * NC>(wv, c.lane);
+    row_allreduce_multi<32, 2 * NL>(wv, c.lane);
 #pragma unroll
-    for (int s = 0; s < NC; ++s) {
-      if (s < S0) continue;
+    for (int j = 0; j < NL; ++j) {
+      const int s = S0 + j;
       const int col = c.gcg + G * s;
       if (col > kk && col < ncol && col != excl) {
-        const float2 tw = X::mul(ct, make_float2(wv[2 * s], wv[2 * s + 1]));
+        const float2 tw = X::mul(ct, make_float2(wv[2 * j], wv[2 * j + 1]));
         upd_slot(v, tw, a, s);
       }
     }

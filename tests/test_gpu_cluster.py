@@ -1,7 +1,8 @@
 """GPU parity of the cluster-per-matrix complex classes (csrc/bqr_cl.cuh:
-`alt_cl4_c64_256x72[_aug]`, `alt_cl2_c64_256x72[_aug]`; one cluster of 4 / 2
-CTAs per matrix, reflectors pushed to every CTA by st.async into distributed
-shared memory).  They are explicit variants (BQR_FORCE_VARIANT, read once per
+`alt_cl4_c64_256x72[_aug]`, `alt_cl2_c64_256x72[_aug]`,
+`alt_cl1_c64_256x72_aug`; one cluster of 4 / 2 / 1 CTAs per matrix,
+reflectors pushed to every CTA by st.async into distributed shared memory,
+or by shared stores + mbarrier arrives on one CTA).  They are explicit variants (BQR_FORCE_VARIANT, read once per
 process), so each runs in a child process that compares geqrf and the fused
 Q^H B against the fp64 oracle (oracle/compare.py, north-star tolerances) and
 prints one JSON line.  Shapes: the STAP shape, the class bound 256 x 72,
@@ -51,7 +52,7 @@ print(json.dumps(res))
 """
 
 
-@pytest.mark.parametrize("variant", ["alt_cl4_c64_256x72_aug", "alt_cl2_c64_256x72_aug"])
+@pytest.mark.parametrize("variant", ["alt_cl4_c64_256x72_aug", "alt_cl2_c64_256x72_aug", "alt_cl1_c64_256x72_aug"])
 def test_cluster_class_parity(variant):
     env = dict(os.environ, BQR_FORCE_VARIANT=variant)
     out = subprocess.run([sys.executable, "-c", f"ROOT = {ROOT!r}\n" + CHILD], env=env, capture_output=True,
