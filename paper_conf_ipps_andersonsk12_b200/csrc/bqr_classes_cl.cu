@@ -66,7 +66,8 @@ const ClassEntry kTable[] = {
     {BQR_C64, 256, 72, 0, 0, true, Plan{"alt_cl4_c64_256x72_aug", &launch_cl<4, 3, 6>, kOrg}},
     {BQR_C64, 256, 72, 0, 0, true, Plan{"alt_cl2_c64_256x72", &launch_cl<2, 6, 6>, kOrg}},
     {BQR_C64, 256, 72, 0, 0, true, Plan{"alt_cl2_c64_256x72_aug", &launch_cl<2, 6, 6>, kOrg}},
-    // the same kernel on one CTA of 12 warps (no distributed shared memory)
+    // the same kernel on one CTA of 12 warps (no distributed shared memory);
+    // 6 / 8 / 16 / 18 / 24 warps per CTA measured slower (c4_cluster.jsonl)
     {BQR_C64, 256, 72, 0, 0, true, Plan{"alt_cl1_c64_256x72_aug", &launch_cl<1, 12, 6>, kOrg}},
 };
 }  // namespace
