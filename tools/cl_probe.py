@@ -64,6 +64,28 @@ for b in (1, 16, 32, 37, 64, 74, 148, 256):
             ts.append(e0.elapsed_time(e1) * 1e3)
     times[b] = round(sorted(ts)[len(ts) // 2], 2)
 row['geqrf_us_noflush' if os.environ.get('CL_PROBE_NOFLUSH') else 'geqrf_us_flushed'] = times
+# the C4 bench step: fused geqrf + Q^H b (one right-hand side) at batch 256
+b = 256
+A0 = torch.randn(b, 66, 240, dtype=torch.complex64, device='cuda')
+B0 = torch.randn(b, 1, 240, dtype=torch.complex64, device='cuda')
+A, Bm = torch.empty_like(A0), torch.empty_like(B0)
+tau = torch.empty(b, 66, dtype=torch.complex64, device='cuda')
+s = torch.cuda.current_stream()
+ts = []
+for it in range(13):
+    A.copy_(A0); Bm.copy_(B0)
+    big.zero_()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(s)
+    st = lib.bqr_geqrf_qhb_batched(bqr.C64, 240, 66, 1, b, ctypes.c_void_p(A.data_ptr()), 240,
+                                   ctypes.c_void_p(tau.data_ptr()), ctypes.c_void_p(Bm.data_ptr()), 240,
+                                   ctypes.c_void_p(s.cuda_stream))
+    e1.record(s)
+    torch.cuda.synchronize()
+    assert st == 0, st
+    if it >= 3:
+        ts.append(e0.elapsed_time(e1) * 1e3)
+row['qhb_256_us_flushed'] = round(sorted(ts)[len(ts) // 2], 2)
 print(json.dumps(row), flush=True)
 """
     env = dict(os.environ)
