@@ -275,3 +275,40 @@ def test_left_looking_kernels_sass(lib):
         assert "BRA.DIV" not in sass and "WARPSYNC" not in sass, mangled
         m = re.search(re.escape(mangled) + r".*?\n\s*REG:(\d+)", res, re.S)
         assert m and int(m.group(1)) <= 96, (mangled, m and m.group(1))
+
+
+def test_cluster_kernels_sass(lib):
+    """The cluster-per-matrix classes (csrc/bqr_cl.cuh): the multi-CTA
+    instantiations publish reflectors with st.async into distributed shared
+    memory (SASS STAS) counted by mbarriers (SYNCS), with no GPU-scope fence
+    on the per-column path (only the per-matrix cluster barrier's); the
+    one-CTA instantiation uses plain shared stores; all use packed FP32
+    (FFMA2) for the complex updates and spill nothing."""
+    import re
+    import shutil
+    import subprocess
+    exe = shutil.which("cuobjdump") or "/usr/local/cuda/bin/cuobjdump"
+    if not os.path.exists(exe):
+        pytest.skip("cuobjdump not available")
+    res = subprocess.run([exe, "-res-usage", bqr._LIB_PATH], capture_output=True, text=True, timeout=600).stdout
+    sass_all = subprocess.run([exe, "-sass", bqr._LIB_PATH], capture_output=True, text=True, timeout=600).stdout
+    funcs = {}
+    fn = None
+    for line in sass_all.splitlines():
+        m = re.search(r"Function : (\S+)", line)
+        if m:
+            fn = m.group(1)
+            funcs.setdefault(fn, [])
+        elif fn:
+            funcs[fn].append(line)
+    cl = {f: "\n".join(v) for f, v in funcs.items() if "geqrf_cl_kernel" in f}
+    assert any("ILi4E" in f for f in cl) and any("ILi2E" in f for f in cl) and any("ILi1E" in f for f in cl), list(cl)
+    for f, sass in cl.items():
+        assert "FFMA2" in sass, f
+        assert "SYNCS" in sass, f
+        assert "LDL" not in sass and "STL" not in sass, f
+        multi = "ILi1E" not in f.split("geqrf_cl_kernel")[1][:6]
+        assert ("STAS" in sass) == multi, f
+        assert sass.count("MEMBAR.ALL.GPU") <= 4, f  # the cluster barriers per matrix only
+        m = re.search(re.escape(f) + r".*?\n\s*REG:\d+ STACK:(\d+)", res, re.S)
+        assert m and int(m.group(1)) == 0, (f, m and m.group(1))
