@@ -6,8 +6,9 @@ or by shared stores + mbarrier arrives on one CTA).  They are explicit variants 
 process), so each runs in a child process that compares geqrf and the fused
 Q^H B against the fp64 oracle (oracle/compare.py, north-star tolerances) and
 prints one JSON line.  Shapes: the STAP shape, the class bound 256 x 72,
-ragged row/column counts, a batch larger than the resident clusters (the
-persistent loop and its ring-phase continuation), several right-hand
+ragged row/column counts, 1 x 1 / 2 x 2 / 256 x 1 matrices (the complex
+1-row reflector), a batch larger than the resident clusters
+(the persistent loop and its ring-phase continuation), several right-hand
 sides."""
 import json
 import os
@@ -35,7 +36,8 @@ lib = bqr.load()
 res = {'kernel': bqr.kernel_name(bqr.C64, 240, 66), 'qhb_kernel': lib.bqr_qhb_kernel_name(bqr.C64, 240, 66, 1).decode(),
        'resident': lib.bqr_resident_matrices(bqr.C64, 240, 66), 'cases': []}
 for m, n, b, seed in ((240, 66, 7, 11), (256, 72, 5, 12), (255, 71, 3, 13), (131, 40, 4, 14), (33, 33, 3, 15),
-                      (240, 66, 2 * res['resident'] + 5, 16)):
+                      (240, 66, 2 * res['resident'] + 5, 16), (1, 1, 3, 17), (2, 2, 3, 18), (256, 1, 3, 19),
+                      (72, 72, 2, 20)):
     A = bqr_inputs.random_batch(m, n, b, 'c64', seed=seed)
     out, tau = geqrf_gpu(A, m)
     idx = sorted(set(range(0, b, max(1, b // 12))) | {b - 1})
